@@ -9,7 +9,10 @@ Every generator is a pure function of (config, seed); numpy default_rng(seed), s
 """
 from __future__ import annotations
 
+import ctypes
 import math
+import os
+import subprocess
 from dataclasses import dataclass, field
 
 import numpy as np
@@ -18,6 +21,26 @@ from .batch import Batch, _ranges_to_ids
 
 ASCII = np.frombuffer(b"ACGTN", np.uint8)
 RL = 150                      # read length (150 bp reads)
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libsynth.so")
+_clib = None
+
+
+def _c():
+    """Seeded C helpers (_synth.c): genome and read synthesis, OpenMP, counter-based RNG."""
+    global _clib
+    if _clib is None:
+        src = os.path.join(_HERE, "_synth.c")
+        if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
+            subprocess.check_call(["gcc", "-O3", "-fopenmp", "-shared", "-fPIC", "-o", _SO, src])
+        lib = ctypes.CDLL(_SO)
+        V = ctypes.c_void_p
+        lib.synth_genome.argtypes = [V, ctypes.c_int64, ctypes.c_double, ctypes.c_uint64]
+        lib.synth_reads.argtypes = [V, V, V, ctypes.c_int64, ctypes.c_int, ctypes.c_uint64, ctypes.c_double,
+                                    ctypes.c_double, V, V]
+        _clib = lib
+    return _clib
 
 
 def seed_for(cfg_index: int) -> int:
@@ -96,9 +119,9 @@ class MetaCfg:
 
 
 def _species_genome(rng, sp: Species) -> np.ndarray:
-    p_gc = sp.gc / 2
-    p_at = (1 - sp.gc) / 2
-    return rng.choice(4, size=sp.length, p=[p_at, p_gc, p_gc, p_at]).astype(np.uint8)
+    g = np.empty(sp.length, np.uint8)
+    _c().synth_genome(g.ctypes.data, sp.length, float(sp.gc), int(rng.integers(0, 2 ** 63)))
+    return g
 
 
 def _intervals(mask: np.ndarray):
@@ -291,24 +314,11 @@ def make_metagenome(cfg: MetaCfg, seed: int, max_contigs: int | None = None) -> 
     U = uniq.shape[0]
     useq = np.empty((U, RL), np.uint8)
     uqual = np.empty((U, RL), np.uint8)
-    CH = 1 << 18
-    ar = np.arange(RL, dtype=np.int64)
-    for c0 in range(0, U, CH):
-        st = ustart[c0:c0 + CH]
-        b = gall[st[:, None] + ar]
-        n = b.shape[0]
-        u = rng.random((n, RL))
-        err = u < cfg.err
-        nn = (u >= cfg.err) & (u < cfg.err + cfg.n_rate)
-        b = np.where(err, (b + rng.integers(1, 4, (n, RL), dtype=np.uint8)) % 4, b)
-        good = rng.random((n, RL)) < 0.9
-        q = np.where(good, rng.integers(30, 41, (n, RL), dtype=np.uint8),
-                     rng.integers(2, 30, (n, RL), dtype=np.uint8))
-        q = np.where(err, rng.integers(2, 26, (n, RL), dtype=np.uint8), q)
-        b = np.where(nn, 4, b)
-        q = np.where(nn, 2, q)
-        useq[c0:c0 + n] = ASCII[b]
-        uqual[c0:c0 + n] = q + 33
+    ustart = np.ascontiguousarray(ustart, np.int64)
+    uniq = np.ascontiguousarray(uniq, np.int64)
+    _c().synth_reads(gall.ctypes.data, ustart.ctypes.data, uniq.ctypes.data, U, RL,
+                     int(rng.integers(0, 2 ** 63)), float(cfg.err), float(cfg.n_rate),
+                     useq.ctypes.data, uqual.ctypes.data)
 
     # assemble the batch
     read_seq = useq[inv].reshape(-1)

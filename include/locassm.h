@@ -1,0 +1,132 @@
+/*
+ * locassm.h — C ABI of the B200 (sm_100a) local-assembly library.
+ *
+ * The operation (paper = /root/reference/PAPER.md, "P:L<line>"):
+ *   MetaHipMer local assembly extends every contig end using only the reads that map to that end
+ *   (§2.3).  For each end: build a k-mer -> extension hash table from the end's
+ *   candidate reads (Alg 1; the value is the following base with its quality and count,
+ *   P:L450-457), then mer-walk from the contig's last k-mer until a dead end, a fork, a loop or
+ *   max_walk_len (Alg 2), and retry with k up-shifted after a fork and down-shifted
+ *   after a dead end, stopping on a fork after a down-shift or a dead end after an up-shift
+ *   (Fig 5).  Reads of the left and right side are kept separate and the same
+ *   algorithm runs on both sides (Fig 4); a left end is computed as the right end of the
+ *   reverse-complement problem and its extension is returned in contig-forward orientation.
+ *   Where the paper is silent the readings listed in DESIGN.md §3 apply (vote rule, quality tiers,
+ *   loop handling, choice of the returned walk, N handling, ...).
+ *
+ * Results are deterministic and equal, per end, to the CPU oracle (oracle/oracle.cpp) bit for bit:
+ * extension string, termination code, k of the returned walk and number of attempts.
+ *
+ * Conventions: every call returns la_status; nothing is thrown across the ABI; no C++ types.
+ * A context is bound to one CUDA device and one stream and is NOT thread-safe.
+ */
+#ifndef LOCASSM_H
+#define LOCASSM_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct la_ctx la_ctx; /* opaque */
+
+typedef enum {
+    LA_OK = 0,
+    LA_ERR_INVALID_ARG = -1, /* bad pointer, offsets, characters, lengths or parameters; the
+                                context is unchanged */
+    LA_ERR_OOM = -2,         /* device or pinned host allocation failed                       */
+    LA_ERR_CUDA = -3,        /* CUDA error; sticky: the caller must la_destroy the context     */
+    LA_ERR_STATE = -4,       /* la_extend before a successful la_load_batch                    */
+    LA_ERR_CAPACITY = -5     /* an internal bound was exceeded (never a silent drop)           */
+} la_status;
+
+typedef enum {
+    LA_TERM_DEADEND = 0, /* lookup found no usable extension (Alg 2 line 10, "end")           */
+    LA_TERM_FORK = 1,    /* two or more candidate extensions (Alg 2 line 10, "fork")          */
+    LA_TERM_LOOP = 2,    /* the next k-mer was already visited in this walk (Alg 2 line 6)    */
+    LA_TERM_MAXLEN = 3,  /* max_walk_len bases appended (Alg 2 line 5 bound)                  */
+    LA_TERM_NOREADS = 4, /* the end has no candidate reads (bin 1): not extended  */
+    LA_TERM_SHORT = 5    /* contig shorter than k_start: no start k-mer                       */
+} la_term;
+
+typedef enum { LA_MEM_HOST = 0, LA_MEM_DEVICE = 1 } la_mem;
+
+typedef struct {
+    int32_t k_start, k_min, k_max, k_shift; /* 1 <= k_min <= k_start <= k_max <= 128; k_shift >= 1 */
+    int32_t max_walk_len;                   /* W: 0 <= W <= 1024 (paper: walks up to 300) */
+    int32_t qual_offset;                    /* Phred offset of read_qual characters, e.g. 33      */
+    int32_t q_lo, q_hi;                     /* 0 <= q_lo <= q_hi <= 93: a base of quality q gives a
+                                               low-tier vote if q >= q_lo and also a high-tier vote
+                                               if q >= q_hi (reading #2)                          */
+    int32_t min_votes;                      /* V >= 1 (reading #3)                                */
+    int32_t min_frac_pct;                   /* F in 0..100 (reading #3)                           */
+} la_params;
+
+/* Input batch.  Caller-owned, read only during la_load_batch, may be freed after it returns.
+ * mem = LA_MEM_HOST: all pointers are host memory (pinned memory is fastest);
+ * mem = LA_MEM_DEVICE: all pointers are device memory of the context's device (e.g. torch tensor
+ * data_ptr()); the loader reads them on the context stream.
+ * Offsets start at 0 and are non-decreasing. */
+typedef struct {
+    int32_t mem;
+    int32_t n_contigs;
+    const char *contig_seq;       /* uppercase A,C,G,T,N                                      */
+    const int64_t *contig_off;    /* [n_contigs+1]                                            */
+    int64_t n_reads;
+    const char *read_seq;         /* A,C,G,T,N; each read in its end's contig-forward orientation */
+    const char *read_qual;        /* one quality character per base, >= qual_offset           */
+    const int64_t *read_off;      /* [n_reads+1]; every read 0 <= len <= 300     */
+    const int64_t *end_read_off;  /* [2*n_contigs+1]; end 2c = LEFT of contig c, 2c+1 = RIGHT;
+                                     end e owns reads end_read_off[e] .. end_read_off[e+1]-1;
+                                     end_read_off[2*n_contigs] == n_reads                       */
+} la_batch;
+
+/* Results.  Library-owned host memory, valid until the next la_load_batch / la_extend /
+ * la_destroy on the same context. */
+typedef struct {
+    int64_t n_ends;               /* 2*n_contigs                                               */
+    const int64_t *ext_off;       /* [n_ends+1]; extension of end e is ext_seq[ext_off[e]..ext_off[e+1]) */
+    const char *ext_seq;          /* LEFT ends: contig-forward orientation, to prepend; RIGHT: to append */
+    const uint8_t *term;          /* la_term of the returned walk                               */
+    const uint8_t *k_used;        /* k of the returned walk (0 for NOREADS / SHORT)             */
+    const uint8_t *n_attempts;    /* number of table builds + walks made for the end            */
+} la_result;
+
+typedef struct {
+    double ms_total;          /* device time of the last la_extend (CUDA events on the ctx stream) */
+    double ms_smem;           /* device time of the shared-memory-table kernel                  */
+    double ms_global;         /* device time of the global-memory-table rounds                  */
+    double ms_emit;           /* device time of result compaction                               */
+    int64_t inserts;          /* sum over attempts of k-mer occurrences with a following base    */
+    int64_t inserts_smem;     /* ... of which made by the shared-memory-table kernel             */
+    int64_t walk_steps;       /* table lookups made by walks                                     */
+    int64_t attempts;         /* table builds                                                    */
+    int64_t ext_bases;        /* total extension length                                          */
+    int64_t ends_by_class[5]; /* NOREADS, SHORT, SMEM, GLOBAL, SMEM->GLOBAL (smem table overflow) */
+    int64_t kernel_launches;  /* kernels launched by the last la_extend                          */
+    int64_t smem_bytes_per_cta;
+    int32_t smem_ctas_per_sm;
+    int32_t global_rounds;
+} la_stats;
+
+la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);
+la_status la_load_batch(la_ctx *ctx, const la_batch *batch, const la_params *params);
+/* Runs the extension on the device and blocks until the results are in host memory. */
+la_status la_extend(la_ctx *ctx, la_result *out);
+/* Same, but leaves the results on the device only (no device-to-host copy); for device-resident
+ * pipelines and the kernel-only benchmark.  Device pointers are returned in *out. */
+la_status la_extend_device(la_ctx *ctx, la_result *out);
+la_status la_get_stats(const la_ctx *ctx, la_stats *out);
+la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
+const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */
+
+/* Host-side helper (no GPU needed): table capacity the planner reserves for an end whose reads
+ * hold `inserts` k-mer occurrences with a following base, and the paper's load-factor bound
+ * (l-k+1)/l for table size l*r.  Exposed for tests. */
+int64_t la_plan_global_capacity(int64_t inserts);
+double la_paper_load_factor(int32_t max_read_len, int32_t k);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

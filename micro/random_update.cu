@@ -1,0 +1,111 @@
+// random_update.cu — microbenchmarks of the roofline denominators:
+// the random-update rate of the memory that holds a k-mer table.
+//   smem_atomic_add : random 32-bit atomicAdd into a per-CTA shared-memory table (ATOMS.ADD)
+//   smem_cas64      : random 64-bit atomicCAS into shared memory (ATOMS.CAS.64)
+//   smem_load64     : random 64-bit loads from shared memory (LDS.64, the probe)
+//   global_red_l2   : random 32-bit atomicAdd (RED.ADD) into a 64 MB L2-resident global table
+//   global_red_hbm  : same into a 4 GB table (HBM-bound)
+// Output: one JSON line, G updates/s per variant (best of 5, CUDA events).
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o micro/random_update micro/random_update.cu
+#include <cuda_runtime.h>
+#include <cstdio>
+#include <cstdint>
+
+__device__ __forceinline__ uint32_t hsh(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+    return x;
+}
+
+template <int MODE>
+__global__ void k_smem(int iters, uint32_t words, unsigned long long *sink) {
+    extern __shared__ uint32_t t[];
+    for (uint32_t i = threadIdx.x; i < words; i += blockDim.x) t[i] = 0;
+    __syncthreads();
+    uint32_t x = hsh(blockIdx.x * 7919u + threadIdx.x);
+    uint64_t acc = 0;
+    for (int it = 0; it < iters; ++it) {
+        x = hsh(x + it);
+        if (MODE == 0) {
+            atomicAdd(&t[x % words], 1u);
+        } else if (MODE == 1) {
+            unsigned long long *t64 = (unsigned long long *)t;
+            acc += atomicCAS(&t64[x % (words / 2)], 0ull, (unsigned long long)x);
+        } else {
+            const unsigned long long *t64 = (const unsigned long long *)t;
+            acc += t64[x % (words / 2)];
+        }
+    }
+    __syncthreads();
+    if (acc == 0x12345678ull) sink[0] = acc + t[threadIdx.x % words];
+}
+
+__global__ void k_global(uint32_t *tab, uint64_t words, int iters) {
+    uint32_t x = hsh(blockIdx.x * 7919u + threadIdx.x);
+    for (int it = 0; it < iters; ++it) {
+        x = hsh(x + it);
+        uint64_t i = ((uint64_t)x * 0x9E3779B1u + it) % words;
+        atomicAdd(&tab[i], 1u);
+    }
+}
+
+int main() {
+    cudaDeviceProp p;
+    cudaGetDeviceProperties(&p, 0);
+    const int sms = p.multiProcessorCount;
+    unsigned long long *sink;
+    cudaMalloc(&sink, 64);
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    const int threads = 256, ctas_per_sm = 2;
+    const uint32_t bytes = 110 * 1024;
+    const uint32_t words = bytes / 4;
+    const int iters = 4096;
+    double res[5] = {0, 0, 0, 0, 0};
+    cudaFuncSetAttribute(k_smem<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(k_smem<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    cudaFuncSetAttribute(k_smem<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    for (int mode = 0; mode < 3; ++mode) {
+        double best = 0;
+        for (int rep = 0; rep < 6; ++rep) {
+            cudaEventRecord(a);
+            if (mode == 0) k_smem<0><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
+            if (mode == 1) k_smem<1><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
+            if (mode == 2) k_smem<2><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
+            cudaEventRecord(b);
+            cudaEventSynchronize(b);
+            float ms;
+            cudaEventElapsedTime(&ms, a, b);
+            double ops = (double)sms * ctas_per_sm * threads * iters;
+            if (rep) best = best > ops / ms / 1e6 ? best : ops / ms / 1e6;
+        }
+        res[mode] = best;
+    }
+    for (int g = 0; g < 2; ++g) {
+        uint64_t words_g = g == 0 ? (64ull << 20) / 4 : (4ull << 30) / 4;
+        uint32_t *tab;
+        if (cudaMalloc(&tab, words_g * 4) != cudaSuccess) continue;
+        cudaMemset(tab, 0, words_g * 4);
+        double best = 0;
+        const int gi = 256;
+        const int grid = sms * 8;
+        for (int rep = 0; rep < 6; ++rep) {
+            cudaEventRecord(a);
+            k_global<<<grid, 256>>>(tab, words_g, gi);
+            cudaEventRecord(b);
+            cudaEventSynchronize(b);
+            float ms;
+            cudaEventElapsedTime(&ms, a, b);
+            double ops = (double)grid * 256 * gi;
+            if (rep) best = best > ops / ms / 1e6 ? best : ops / ms / 1e6;
+        }
+        res[3 + g] = best;
+        cudaFree(tab);
+    }
+    printf("{\"unit\": \"G updates/s\", \"smem_atomic_add\": %.2f, \"smem_cas64\": %.2f, \"smem_load64\": %.2f, "
+           "\"global_red_l2\": %.2f, \"global_red_hbm\": %.2f, \"sms\": %d, \"smem_ctas_per_sm\": %d, "
+           "\"threads\": %d, \"smem_bytes_per_cta\": %u, \"err\": \"%s\"}\n",
+           res[0], res[1], res[2], res[3], res[4], sms, ctas_per_sm, threads, bytes,
+           cudaGetErrorString(cudaGetLastError()));
+    return 0;
+}

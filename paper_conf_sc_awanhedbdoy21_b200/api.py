@@ -1,0 +1,147 @@
+"""Python face of the C ABI: `LocalAssembler` (one context per device/stream).
+
+Argument marshalling only — every step of the path (validation, encoding, planning, table build,
+walk, retry, compaction) runs in the CUDA library.  Inputs may be numpy arrays (host) or torch
+tensors (host, pinned or CUDA); a batch is any object with the attributes contig_seq, contig_off,
+read_seq, read_qual, read_off, end_read_off (uint8 / int64 arrays in the layout of locassm.h).
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _lib as L
+
+PARAM_FIELDS = ("k_start", "k_min", "k_max", "k_shift", "max_walk_len", "qual_offset", "q_lo",
+                "q_hi", "min_votes", "min_frac_pct")
+DEFAULTS = dict(k_start=33, k_min=21, k_max=99, k_shift=8, max_walk_len=300, qual_offset=33,
+                q_lo=10, q_hi=20, min_votes=2, min_frac_pct=20)
+
+
+def _params(p) -> L.la_params:
+    if p is None:
+        p = DEFAULTS
+    get = (lambda n: p[n]) if isinstance(p, dict) else (lambda n: getattr(p, n))
+    return L.la_params(*[int(get(n)) for n in PARAM_FIELDS])
+
+
+def _ptr_and_mem(a):
+    """(pointer, is_device, keepalive) of a numpy array or torch tensor."""
+    try:
+        import torch
+        if isinstance(a, torch.Tensor):
+            a = a.contiguous()
+            return a.data_ptr(), a.is_cuda, a
+    except ImportError:  # pragma: no cover
+        pass
+    a = np.ascontiguousarray(a)
+    return a.ctypes.data, False, a
+
+
+@dataclass
+class Result:
+    ext_off: np.ndarray
+    ext_seq: np.ndarray      # uint8 ASCII
+    term: np.ndarray
+    k_used: np.ndarray
+    n_attempts: np.ndarray
+
+    @property
+    def n_ends(self):
+        return self.term.shape[0]
+
+    def ext(self, e: int) -> str:
+        return self.ext_seq[self.ext_off[e]:self.ext_off[e + 1]].tobytes().decode()
+
+    def ext_list(self):
+        b = self.ext_seq.tobytes()
+        o = self.ext_off
+        return [b[o[i]:o[i + 1]].decode() for i in range(self.n_ends)]
+
+
+class LocalAssembler:
+    """la_create / la_load_batch / la_extend / la_destroy."""
+
+    def __init__(self, device: int = 0, stream=None):
+        self._lib = L.load()
+        self._ctx = ctypes.c_void_p()
+        sp = None
+        if stream is not None:
+            sp = stream if isinstance(stream, int) else getattr(stream, "cuda_stream", None)
+        st = self._lib.la_create(ctypes.byref(self._ctx), int(device), ctypes.c_void_p(sp) if sp else None)
+        if st != L.LA_OK:
+            raise L.LocAssmError(st, "la_create failed (no CUDA device?)")
+        self._keep = None
+
+    def _check(self, st):
+        if st != L.LA_OK:
+            raise L.LocAssmError(st, self._lib.la_last_error(self._ctx).decode())
+
+    def load(self, batch, params=None):
+        arrs = [batch.contig_seq, batch.contig_off, batch.read_seq, batch.read_qual, batch.read_off,
+                batch.end_read_off]
+        ptrs, devs, keep = zip(*[_ptr_and_mem(a) for a in arrs])
+        if len(set(devs)) != 1:
+            raise ValueError("batch arrays must all be host or all be device memory")
+        n_contigs = int(arrs[1].shape[0]) - 1
+        n_reads = int(arrs[4].shape[0]) - 1
+        b = L.la_batch(L.LA_MEM_DEVICE if devs[0] else L.LA_MEM_HOST, n_contigs, ptrs[0], ptrs[1], n_reads,
+                       ptrs[2], ptrs[3], ptrs[4], ptrs[5])
+        p = _params(params)
+        self._check(self._lib.la_load_batch(self._ctx, ctypes.byref(b), ctypes.byref(p)))
+        self._keep = keep
+        return self
+
+    def extend(self) -> Result:
+        r = L.la_result()
+        self._check(self._lib.la_extend(self._ctx, ctypes.byref(r)))
+        n = int(r.n_ends)
+
+        def arr(ptr, count, dtype):
+            if count == 0:
+                return np.zeros(0, dtype)
+            buf = (ctypes.c_char * (count * np.dtype(dtype).itemsize)).from_address(ptr)
+            return np.frombuffer(buf, dtype=dtype, count=count).copy()
+
+        off = arr(r.ext_off, n + 1, np.int64)
+        return Result(off, arr(r.ext_seq, int(off[-1]) if n else 0, np.uint8), arr(r.term, n, np.uint8),
+                      arr(r.k_used, n, np.uint8), arr(r.n_attempts, n, np.uint8))
+
+    def extend_device(self) -> dict:
+        """Run without copying results to the host; returns device pointers (valid until the next call)."""
+        r = L.la_result()
+        self._check(self._lib.la_extend_device(self._ctx, ctypes.byref(r)))
+        return dict(n_ends=int(r.n_ends), ext_off=r.ext_off, ext_seq=r.ext_seq, term=r.term,
+                    k_used=r.k_used, n_attempts=r.n_attempts)
+
+    def stats(self) -> dict:
+        s = L.la_stats()
+        self._check(self._lib.la_get_stats(self._ctx, ctypes.byref(s)))
+        d = {f: getattr(s, f) for f, _ in L.la_stats._fields_}
+        d["ends_by_class"] = list(s.ends_by_class)
+        return d
+
+    def close(self):
+        if getattr(self, "_ctx", None) and self._ctx.value:
+            self._lib.la_destroy(self._ctx)
+            self._ctx = ctypes.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def extend(batch, params=None, device: int = 0) -> Result:
+    """One-shot convenience: create, load, extend, destroy."""
+    with LocalAssembler(device) as la:
+        return la.load(batch, params).extend()

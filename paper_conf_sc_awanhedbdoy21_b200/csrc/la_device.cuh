@@ -1,0 +1,140 @@
+// la_device.cuh — device-side building blocks of the sm_100a local-assembly path.
+//
+// Encodings (DESIGN.md §6 "Data layout in HBM"):
+//  * bases: 2 bits (A0 C1 G2 T3), big-endian inside u64 words: base i of a read sits in word i/32
+//    at bit 62 - 2*(i%32).  Every read owns SW words (zero padded) in `rseq`.
+//  * quality class, same layout in `rqc`: 0 = no vote (q < q_lo), 1 = low-tier vote
+//    (q_lo <= q < q_hi), 2 = both tiers (q >= q_hi), 3 = the base is N (reading #2, #5).
+//  * k-mers: KW = ceil(2k/64) u64 words, left aligned (base 0 in the top bits of word 0), the
+//    2*(32*KW-k) low bits of the last word zero.
+//  * table slot: u64 = tag(23) | read(32) | pos(9); 0 = empty.  The key is NOT stored: it is the
+//    k-mer of read `read` at `pos` (pointer-encoded key, Fig 6), verified against the
+//    packed read on every tag match, so equality is exact.
+#pragma once
+#include <cstdint>
+
+namespace la {
+
+constexpr int MAX_KW = 4;            // k <= 128
+constexpr int MAX_READ_LEN = 300;
+constexpr uint32_t NONE = 0x1FFFFFFFu;
+enum : int { CODE_FORK = 4, CODE_DEADEND = 5 };
+enum : int { T_DEADEND = 0, T_FORK = 1, T_LOOP = 2, T_MAXLEN = 3, T_NOREADS = 4, T_SHORT = 5 };
+
+struct DevParams {
+    int k_start, k_min, k_max, k_shift, W, qual_offset, q_lo, q_hi, V, F;
+};
+
+__host__ __device__ __forceinline__ int kwords(int k) { return (2 * k + 63) >> 6; }
+
+struct Kmer {
+    uint64_t w[MAX_KW];
+};
+
+__device__ __forceinline__ uint64_t funnel64(uint64_t hi, uint64_t lo, int s) {
+    return s ? ((hi << s) | (lo >> (64 - s))) : hi;
+}
+
+// k-mer of length k starting at base p of the packed sequence R (words in any address space).
+template <typename P>
+__device__ __forceinline__ Kmer extract_kmer(const P *R, int p, int k, int KW) {
+    Kmer K;
+    const int q = p >> 5, s = (p & 31) << 1;
+#pragma unroll
+    for (int w = 0; w < MAX_KW; ++w) {
+        if (w < KW) K.w[w] = funnel64(R[q + w], R[q + w + 1], s);
+        else K.w[w] = 0;
+    }
+    const int pad = 64 * KW - 2 * k;
+#pragma unroll
+    for (int w = 0; w < MAX_KW; ++w)
+        if (w == KW - 1 && pad) K.w[w] &= (~0ull) << pad;
+    return K;
+}
+
+// next_kmer (Alg 2 line 15): drop base 0, append base b.
+__device__ __forceinline__ void roll_kmer(Kmer &K, int k, int KW, uint32_t b) {
+#pragma unroll
+    for (int w = 0; w < MAX_KW; ++w) {
+        if (w < KW - 1) K.w[w] = (K.w[w] << 2) | (K.w[w + 1] >> 62);
+        else if (w == KW - 1) K.w[w] = (K.w[w] << 2) | ((uint64_t)b << (64 * KW - 2 * k));
+    }
+}
+
+__device__ __forceinline__ bool kmer_eq(const Kmer &a, const Kmer &b, int KW) {
+    bool eq = true;
+#pragma unroll
+    for (int w = 0; w < MAX_KW; ++w)
+        if (w < KW) eq &= (a.w[w] == b.w[w]);
+    return eq;
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t x) {
+    x ^= x >> 30;
+    x *= 0xbf58476d1ce4e5b9ull;
+    x ^= x >> 27;
+    x *= 0x94d049bb133111ebull;
+    x ^= x >> 31;
+    return x;
+}
+
+// Hash of a k-mer; the hash function does not affect results (reading #17).
+__device__ __forceinline__ uint64_t hash_kmer(const Kmer &K, int KW) {
+    uint64_t h = 0x9E3779B97F4A7C15ull;
+#pragma unroll
+    for (int w = 0; w < MAX_KW; ++w)
+        if (w < KW) h = mix64(h ^ K.w[w]);
+    return h;
+}
+
+__device__ __forceinline__ uint32_t slot_of(uint64_t h, uint32_t cap) {
+    return (uint32_t)(((uint64_t)(uint32_t)h * cap) >> 32);
+}
+__device__ __forceinline__ uint64_t tag_of(uint64_t h) { return ((h >> 41) | 1ull) << 41; }
+__device__ __forceinline__ uint64_t make_slot(uint64_t tag, uint32_t read, uint32_t pos) {
+    return tag | ((uint64_t)read << 9) | pos;
+}
+__device__ __forceinline__ uint32_t slot_read(uint64_t w) { return (uint32_t)(w >> 9); }
+__device__ __forceinline__ uint32_t slot_pos(uint64_t w) { return (uint32_t)(w & 511u); }
+constexpr uint64_t TAG_MASK = ~((1ull << 41) - 1);
+
+__device__ __forceinline__ uint32_t get2(const uint64_t *R, int i) {
+    return (uint32_t)(R[i >> 5] >> (62 - ((i & 31) << 1))) & 3u;
+}
+
+// Reading #1: two-tier vote rule on exact integer counts.  Returns 0..3 (base), CODE_FORK or
+// CODE_DEADEND.
+__device__ __forceinline__ int ext_rule(const uint32_t lo[4], const uint32_t hi[4], int V, int F) {
+    uint64_t H = (uint64_t)hi[0] + hi[1] + hi[2] + hi[3];
+    uint64_t L = (uint64_t)lo[0] + lo[1] + lo[2] + lo[3];
+    int n = 0, pick = 0;
+#pragma unroll
+    for (int b = 0; b < 4; ++b)
+        if (hi[b] >= (uint32_t)V && 100ull * hi[b] >= (uint64_t)F * H) { ++n; pick = b; }
+    if (n == 1) return pick;
+    if (n >= 2) return CODE_FORK;
+    n = 0;
+#pragma unroll
+    for (int b = 0; b < 4; ++b)
+        if (lo[b] >= (uint32_t)V && 100ull * lo[b] >= (uint64_t)F * L) { ++n; pick = b; }
+    if (n == 1) return pick;
+    if (n >= 2) return CODE_FORK;
+    return CODE_DEADEND;
+}
+
+// The k up/down-shift rule (readings #8, #10).  Returns true when the end is done,
+// else updates k / shift for the next attempt.
+__device__ __forceinline__ bool next_k(int term, int &k, int &shift, int kmax_eff, const DevParams &P) {
+    if (term == T_MAXLEN) return true;
+    if (term == T_DEADEND) {
+        if (shift > 0) return true;
+        shift = -P.k_shift;
+    } else {
+        if (shift < 0) return true;
+        shift = P.k_shift;
+    }
+    k += shift;
+    return k < P.k_min || k > kmax_eff;
+}
+
+}  // namespace la

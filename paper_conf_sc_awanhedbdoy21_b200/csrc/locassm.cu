@@ -1,0 +1,628 @@
+// locassm.cu — the C ABI (include/locassm.h) and the host-side runtime of the sm_100a local-assembly
+// library: context, validation + encode on load, planning, launches, result compaction.
+//
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -shared -Xcompiler -fPIC
+// (see paper_conf_sc_awanhedbdoy21_b200/build.py).  No torch types cross this boundary.
+#include <cuda_runtime.h>
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "locassm.h"
+#include "la_kernels.cuh"
+
+using namespace la;
+
+namespace {
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t n = 0;
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+};
+
+struct HostBuf {
+    void *p = nullptr;
+    size_t n = 0;
+    void release() {
+        if (p) cudaFreeHost(p);
+        p = nullptr;
+        n = 0;
+    }
+};
+
+// Encoded batch (device), produced by la_load_batch.
+struct Encoded {
+    int64_t n_contigs = 0, n_ends = 0, n_reads = 0;
+    int SW = 2, maxlen = 0;
+    DevBuf eoff, roff, rseq, rqc, rlen, rflag, tail, tailN, clen;
+    void release() {
+        for (DevBuf *b : {&eoff, &roff, &rseq, &rqc, &rlen, &rflag, &tail, &tailN, &clen}) b->release();
+    }
+};
+
+}  // namespace
+
+struct la_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    bool sticky = false;
+    bool loaded = false;
+    std::string err;
+    int n_sm = 148;
+    int smem_ctas_per_sm = 2;
+    uint32_t smem_bytes = 0;
+    la_params params{};
+    DevParams dp{};
+    Encoded enc, spare;   // current encoding; la_load_batch fills `spare` and swaps on success
+    // scratch (grow-only)
+    DevBuf raw_seq, raw_qual, raw_coff, raw_cseq, read_end, errw;
+    DevBuf cls, out_len, out_term, out_k, out_att, walk_buf, smem_list, smem_key, smem_list2,
+        smem_key2, glob_list, ctrs, ext_off, ext_seq, gstats, cub_tmp;
+    DevBuf g_state, g_act, g_act2, g_still, g_cap, g_nrd, g_capoff, g_rdoff, g_slots, g_cnt, g_vis,
+        g_cur;
+    DevBuf lens64;
+    HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
+    int64_t g_attempts = 0;
+    cudaEvent_t ev[6] = {};
+    la_stats stats{};
+};
+
+namespace {
+
+la_status fail(la_ctx *c, la_status s, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) {
+        c->err = buf;
+        if (s == LA_ERR_CUDA) c->sticky = true;
+    }
+    return s;
+}
+
+#define CK(call)                                                                              \
+    do {                                                                                      \
+        cudaError_t _e = (call);                                                              \
+        if (_e != cudaSuccess)                                                                \
+            return fail(ctx, _e == cudaErrorMemoryAllocation ? LA_ERR_OOM : LA_ERR_CUDA,      \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(_e), __FILE__,     \
+                        __LINE__);                                                            \
+    } while (0)
+
+#define CKL()                                                                                 \
+    do {                                                                                      \
+        ctx->stats.kernel_launches++;                                                         \
+        cudaError_t _e = cudaGetLastError();                                                  \
+        if (_e != cudaSuccess)                                                                \
+            return fail(ctx, LA_ERR_CUDA, "kernel launch failed: %s (%s:%d)",                 \
+                        cudaGetErrorString(_e), __FILE__, __LINE__);                          \
+    } while (0)
+
+cudaError_t grow(DevBuf &b, size_t bytes) {
+    if (bytes <= b.n && b.p) return cudaSuccess;
+    b.release();
+    size_t n = std::max<size_t>(bytes, 256);
+    cudaError_t e = cudaMalloc(&b.p, n);
+    if (e == cudaSuccess) b.n = n;
+    else b.p = nullptr;
+    return e;
+}
+
+cudaError_t grow_host(HostBuf &b, size_t bytes) {
+    if (bytes <= b.n && b.p) return cudaSuccess;
+    b.release();
+    size_t n = std::max<size_t>(bytes, 256);
+    cudaError_t e = cudaMallocHost(&b.p, n);
+    if (e == cudaSuccess) b.n = n;
+    else b.p = nullptr;
+    return e;
+}
+
+template <typename T>
+T *P(DevBuf &b) { return (T *)b.p; }
+
+bool valid_params(const la_params &p, std::string &why) {
+    char buf[256];
+    if (!(p.k_min >= 1 && p.k_min <= p.k_start && p.k_start <= p.k_max && p.k_max <= 128)) {
+        snprintf(buf, sizeof buf, "k schedule must satisfy 1 <= k_min <= k_start <= k_max <= 128 (got %d %d %d)",
+                 p.k_min, p.k_start, p.k_max);
+        why = buf;
+        return false;
+    }
+    if (p.k_shift < 1) { why = "k_shift must be >= 1"; return false; }
+    if (p.max_walk_len < 0 || p.max_walk_len > 1024) { why = "max_walk_len must be in 0..1024"; return false; }
+    if (p.qual_offset < 0 || p.qual_offset > 127) { why = "qual_offset must be in 0..127"; return false; }
+    if (!(p.q_lo >= 0 && p.q_lo <= p.q_hi && p.q_hi <= 93)) { why = "need 0 <= q_lo <= q_hi <= 93"; return false; }
+    if (p.min_votes < 1) { why = "min_votes must be >= 1"; return false; }
+    if (p.min_frac_pct < 0 || p.min_frac_pct > 100) { why = "min_frac_pct must be in 0..100"; return false; }
+    return true;
+}
+
+inline unsigned blocks(int64_t n, int b) { return (unsigned)((n + b - 1) / b); }
+
+}  // namespace
+
+// ================================================================================================
+extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
+    if (!out) return LA_ERR_INVALID_ARG;
+    *out = nullptr;
+    la_ctx *ctx = new la_ctx();
+    ctx->device = device;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        delete ctx;
+        return LA_ERR_CUDA;
+    }
+    if (device < 0 || device >= ndev) { delete ctx; return LA_ERR_INVALID_ARG; }
+    if (cudaSetDevice(device) != cudaSuccess) { delete ctx; return LA_ERR_CUDA; }
+    cudaDeviceProp prop;
+    cudaGetDeviceProperties(&prop, device);
+    ctx->n_sm = prop.multiProcessorCount;
+    if (const char *s = getenv("LA_SMEM_CTAS")) ctx->smem_ctas_per_sm = std::max(1, atoi(s));
+    // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
+    size_t per = prop.sharedMemPerMultiprocessor / ctx->smem_ctas_per_sm - 1024 - 512 /* static */;
+    per = std::min(per, (size_t)prop.sharedMemPerBlockOptin);
+    ctx->smem_bytes = (uint32_t)(per & ~(size_t)127);
+    if (cuda_stream) ctx->stream = (cudaStream_t)cuda_stream;
+    else {
+        if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) {
+            delete ctx;
+            return LA_ERR_CUDA;
+        }
+        ctx->own_stream = true;
+    }
+    for (auto &e : ctx->ev) cudaEventCreate(&e);
+    if (cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->smem_bytes) !=
+        cudaSuccess) {
+        cudaGetLastError();
+        la_destroy(ctx);
+        return LA_ERR_CUDA;
+    }
+    *out = ctx;
+    return LA_OK;
+}
+
+extern "C" la_status la_destroy(la_ctx *ctx) {
+    if (!ctx) return LA_OK;
+    cudaSetDevice(ctx->device);
+    if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    ctx->enc.release();
+    ctx->spare.release();
+    for (DevBuf *b : {&ctx->raw_seq, &ctx->raw_qual, &ctx->raw_coff, &ctx->raw_cseq, &ctx->read_end,
+                      &ctx->errw, &ctx->cls, &ctx->out_len, &ctx->out_term, &ctx->out_k, &ctx->out_att,
+                      &ctx->walk_buf, &ctx->smem_list, &ctx->smem_key, &ctx->smem_list2, &ctx->smem_key2,
+                      &ctx->glob_list, &ctx->ctrs, &ctx->ext_off, &ctx->ext_seq, &ctx->gstats,
+                      &ctx->cub_tmp, &ctx->g_state, &ctx->g_act, &ctx->g_act2, &ctx->g_still, &ctx->g_cap,
+                      &ctx->g_nrd, &ctx->g_capoff, &ctx->g_rdoff, &ctx->g_slots, &ctx->g_cnt, &ctx->g_vis,
+                      &ctx->g_cur, &ctx->lens64})
+        b->release();
+    for (HostBuf *b : {&ctx->h_ext_off, &ctx->h_ext_seq, &ctx->h_term, &ctx->h_k, &ctx->h_att, &ctx->h_small})
+        b->release();
+    for (auto &e : ctx->ev)
+        if (e) cudaEventDestroy(e);
+    if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+    delete ctx;
+    return LA_OK;
+}
+
+extern "C" const char *la_last_error(const la_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+extern "C" la_status la_get_stats(const la_ctx *ctx, la_stats *out) {
+    if (!ctx || !out) return LA_ERR_INVALID_ARG;
+    *out = ctx->stats;
+    return LA_OK;
+}
+
+extern "C" int64_t la_plan_global_capacity(int64_t inserts) { return global_capacity(inserts); }
+extern "C" double la_paper_load_factor(int32_t l, int32_t k) { return (double)(l - k + 1) / (double)l; }
+
+// ================================================================================================
+// la_load_batch: copy (if host), validate and encode on the device
+// ================================================================================================
+namespace {
+
+la_status copy_in(la_ctx *ctx, DevBuf &dst, const void *src, size_t bytes, bool host) {
+    CK(grow(dst, bytes + 16));
+    if (bytes) CK(cudaMemcpyAsync(dst.p, src, bytes, host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice,
+                                  ctx->stream));
+    return LA_OK;
+}
+
+la_status read_i64(la_ctx *ctx, const int64_t *p, bool host, int64_t *v) {
+    if (host) { *v = *p; return LA_OK; }
+    CK(cudaMemcpyAsync(v, p, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return LA_OK;
+}
+
+}  // namespace
+
+extern "C" la_status la_load_batch(la_ctx *ctx, const la_batch *b, const la_params *params) {
+    if (!ctx) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
+    if (!b || !params) return fail(ctx, LA_ERR_INVALID_ARG, "null batch or params");
+    std::string why;
+    if (!valid_params(*params, why)) return fail(ctx, LA_ERR_INVALID_ARG, "%s", why.c_str());
+    if (b->mem != LA_MEM_HOST && b->mem != LA_MEM_DEVICE) return fail(ctx, LA_ERR_INVALID_ARG, "bad mem kind");
+    if (b->n_contigs < 0 || b->n_reads < 0) return fail(ctx, LA_ERR_INVALID_ARG, "negative sizes");
+    if (b->n_reads >= (1ll << 32)) return fail(ctx, LA_ERR_INVALID_ARG, "more than 2^32 reads");
+    if (!b->contig_off || !b->read_off || !b->end_read_off)
+        return fail(ctx, LA_ERR_INVALID_ARG, "null offsets array");
+    cudaSetDevice(ctx->device);
+    const bool host = b->mem == LA_MEM_HOST;
+    const int64_t nC = b->n_contigs, nE = 2 * nC, nR = b->n_reads;
+    int64_t c0, cN, r0, rN, e0, eN;
+    la_status s;
+    if ((s = read_i64(ctx, b->contig_off, host, &c0)) || (s = read_i64(ctx, b->contig_off + nC, host, &cN)) ||
+        (s = read_i64(ctx, b->read_off, host, &r0)) || (s = read_i64(ctx, b->read_off + nR, host, &rN)) ||
+        (s = read_i64(ctx, b->end_read_off, host, &e0)) || (s = read_i64(ctx, b->end_read_off + nE, host, &eN)))
+        return s;
+    if (c0 != 0 || r0 != 0 || e0 != 0) return fail(ctx, LA_ERR_INVALID_ARG, "offsets must start at 0");
+    if (cN < 0 || rN < 0) return fail(ctx, LA_ERR_INVALID_ARG, "negative total length");
+    if (eN != nR) return fail(ctx, LA_ERR_INVALID_ARG, "end_read_off[2*n_contigs] (%lld) != n_reads (%lld)",
+                              (long long)eN, (long long)nR);
+    if (rN > (int64_t)nR * MAX_READ_LEN) return fail(ctx, LA_ERR_INVALID_ARG, "reads longer than 300 bases");
+    if ((cN && !b->contig_seq) || (rN && (!b->read_seq || !b->read_qual)))
+        return fail(ctx, LA_ERR_INVALID_ARG, "null sequence pointer");
+
+    Encoded &E = ctx->spare;   // swapped into ctx->enc only if valid (context unchanged on error)
+    E.n_contigs = nC;
+    E.n_ends = nE;
+    E.n_reads = nR;
+    const la_status ok = [&]() -> la_status {
+        cudaStream_t st = ctx->stream;
+        la_status s2;
+        // raw inputs on the device
+        const char *d_seq, *d_qual, *d_cseq;
+        const int64_t *d_coff;
+        CK(grow(E.eoff, (nE + 1) * 8));
+        CK(grow(E.roff, (nR + 1) * 8));
+        CK(cudaMemcpyAsync(E.eoff.p, b->end_read_off, (nE + 1) * 8,
+                           host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(E.roff.p, b->read_off, (nR + 1) * 8,
+                           host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, st));
+        if (host) {
+            if ((s2 = copy_in(ctx, ctx->raw_seq, b->read_seq, rN, true))) return s2;
+            if ((s2 = copy_in(ctx, ctx->raw_qual, b->read_qual, rN, true))) return s2;
+            if ((s2 = copy_in(ctx, ctx->raw_cseq, b->contig_seq, cN, true))) return s2;
+            if ((s2 = copy_in(ctx, ctx->raw_coff, b->contig_off, (nC + 1) * 8, true))) return s2;
+            d_seq = P<char>(ctx->raw_seq);
+            d_qual = P<char>(ctx->raw_qual);
+            d_cseq = P<char>(ctx->raw_cseq);
+            d_coff = P<int64_t>(ctx->raw_coff);
+        } else {
+            d_seq = b->read_seq;
+            d_qual = b->read_qual;
+            d_cseq = b->contig_seq;
+            d_coff = b->contig_off;
+        }
+        // offsets + max read length
+        CK(grow(ctx->errw, 64));
+        uint32_t *d_err = P<uint32_t>(ctx->errw);
+        int *d_maxlen = (int *)(d_err + 1);
+        CK(cudaMemsetAsync(d_err, 0, 8, st));
+        if (nC) { k_check_offsets<<<blocks(nC, 256), 256, 0, st>>>(d_coff, nC, 0, d_err, nullptr); CKL(); }
+        if (nE) { k_check_offsets<<<blocks(nE, 256), 256, 0, st>>>(P<int64_t>(E.eoff), nE, 0, d_err, nullptr); CKL(); }
+        if (nR) { k_check_offsets<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(E.roff), nR, 1, d_err, d_maxlen); CKL(); }
+        uint32_t hv[2] = {0, 0};
+        CK(cudaMemcpyAsync(hv, d_err, 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (hv[0] & ERR_OFFSETS) return fail(ctx, LA_ERR_INVALID_ARG, "offsets are not non-decreasing");
+        if (hv[0] & ERR_READ_LEN) return fail(ctx, LA_ERR_INVALID_ARG, "a read is longer than 300 bases");
+        const int maxlen = (int)hv[1];
+        int SW = (maxlen + 31) / 32 + 2;
+        SW = (SW + 1) & ~1;   // even: 16 B aligned rows
+        E.SW = SW;
+        E.maxlen = maxlen;
+        // encode reads
+        CK(grow(ctx->read_end, std::max<int64_t>(nR, 1) * 4));
+        CK(grow(E.rseq, std::max<int64_t>(nR, 1) * SW * 8));
+        CK(grow(E.rqc, std::max<int64_t>(nR, 1) * SW * 8));
+        CK(grow(E.rlen, std::max<int64_t>(nR, 1) * 2 + 16));
+        CK(grow(E.rflag, std::max<int64_t>(nR, 1) + 16));
+        CK(grow(E.tail, std::max<int64_t>(nE, 1) * TAIL_W * 8));
+        CK(grow(E.tailN, std::max<int64_t>(nE, 1) * 16));
+        CK(grow(E.clen, std::max<int64_t>(nE, 1) * 4));
+        DevParams dp{params->k_start, params->k_min, params->k_max, params->k_shift, params->max_walk_len,
+                     params->qual_offset, params->q_lo, params->q_hi, params->min_votes, params->min_frac_pct};
+        if (nR) {
+            CK(cudaMemsetAsync(E.rflag.p, 0, nR, st));
+            k_read_end<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(E.eoff), nE, nR, P<int32_t>(ctx->read_end));
+            CKL();
+            k_encode_reads<<<blocks(nR * SW, 256), 256, 0, st>>>(
+                d_seq, d_qual, P<int64_t>(E.roff), P<int32_t>(ctx->read_end), nR, SW, dp, P<uint64_t>(E.rseq),
+                P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), d_err);
+            CKL();
+        }
+        if (cN) { k_check_contigs<<<blocks(cN, 256), 256, 0, st>>>(d_cseq, cN, d_err); CKL(); }
+        if (nE) {
+            k_encode_tails<<<blocks(nE, 128), 128, 0, st>>>(d_cseq, d_coff, nE, P<uint64_t>(E.tail),
+                                                            P<uint64_t>(E.tailN), P<int32_t>(E.clen));
+            CKL();
+        }
+        CK(cudaMemcpyAsync(hv, d_err, 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (hv[0] & ERR_READ_CHAR) return fail(ctx, LA_ERR_INVALID_ARG, "read base outside ACGTN");
+        if (hv[0] & ERR_QUAL_CHAR) return fail(ctx, LA_ERR_INVALID_ARG, "quality character below qual_offset");
+        if (hv[0] & ERR_CONTIG_CHAR) return fail(ctx, LA_ERR_INVALID_ARG, "contig base outside ACGTN");
+        ctx->dp = dp;
+        return LA_OK;
+    }();
+    if (ok != LA_OK) return ok;
+    std::swap(ctx->enc, ctx->spare);
+    ctx->params = *params;
+    ctx->loaded = true;
+    return LA_OK;
+}
+
+// ================================================================================================
+// la_extend
+// ================================================================================================
+namespace {
+
+la_status run_global(la_ctx *ctx, const int32_t *d_list, int n_list, double *ms_unused) {
+    (void)ms_unused;
+    cudaStream_t st = ctx->stream;
+    Encoded &E = ctx->enc;
+    const DevParams &dp = ctx->dp;
+    if (n_list == 0) return LA_OK;
+    CK(grow(ctx->g_state, (size_t)n_list * sizeof(GState)));
+    CK(grow(ctx->g_act, (size_t)n_list * 4));
+    CK(grow(ctx->g_act2, (size_t)n_list * 4));
+    CK(grow(ctx->g_still, (size_t)n_list * 4));
+    CK(grow(ctx->g_cap, (size_t)(n_list + 1) * 8));
+    CK(grow(ctx->g_nrd, (size_t)(n_list + 1) * 8));
+    CK(grow(ctx->g_capoff, (size_t)(n_list + 1) * 8));
+    CK(grow(ctx->g_rdoff, (size_t)(n_list + 1) * 8));
+    CK(grow(ctx->g_cur, (size_t)n_list * std::max(dp.W, 1)));
+    GState *gs = P<GState>(ctx->g_state);
+    k_g_init<<<blocks(n_list, 256), 256, 0, st>>>(d_list, n_list, P<int32_t>(E.clen), dp, gs, P<int32_t>(ctx->g_act));
+    CKL();
+    int *d_ctr = P<int>(ctx->ctrs) + 8;
+    unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
+    int n_act = n_list;
+    const int nseg = std::max(1, (E.maxlen - dp.k_min + GSEG - 1) / GSEG);   // positions per read
+    int64_t *h = (int64_t *)ctx->h_small.p;
+    while (n_act > 0) {
+        ctx->stats.global_rounds++;
+        int32_t *act = P<int32_t>(ctx->g_act);
+        k_g_caps<<<n_act, 256, 0, st>>>(act, n_act, d_list, gs, P<int64_t>(E.eoff), P<uint16_t>(E.rlen),
+                                        P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_nrd));
+        CKL();
+        size_t tb = 0;
+        cub::DeviceScan::ExclusiveSum(nullptr, tb, P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_capoff), n_act + 1, st);
+        CK(grow(ctx->cub_tmp, tb));
+        // the element past the end is 0 -> offsets[n] = total
+        CK(cudaMemsetAsync(P<int64_t>(ctx->g_cap) + n_act, 0, 8, st));
+        CK(cudaMemsetAsync(P<int64_t>(ctx->g_nrd) + n_act, 0, 8, st));
+        CK(cudaGetLastError());
+        cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_capoff), n_act + 1, st);
+        CKL();
+        cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->g_nrd), P<int64_t>(ctx->g_rdoff), n_act + 1, st);
+        CKL();
+        CK(cudaMemcpyAsync(h, P<int64_t>(ctx->g_capoff) + n_act, 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h + 1, P<int64_t>(ctx->g_rdoff) + n_act, 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        const int64_t total = h[0], nrd = h[1];
+        if (total >= (int64_t)NONE) return fail(ctx, LA_ERR_CAPACITY, "global table round too large (%lld slots)", (long long)total);
+        CK(grow(ctx->g_slots, (size_t)total * 8));
+        CK(grow(ctx->g_cnt, (size_t)total * 32));
+        const size_t visw = (size_t)(total >> 5) + n_act + 2;
+        CK(grow(ctx->g_vis, visw * 4));
+        CK(cudaMemsetAsync(ctx->g_slots.p, 0, (size_t)total * 8, st));
+        CK(cudaMemsetAsync(ctx->g_cnt.p, 0, (size_t)total * 32, st));
+        CK(cudaMemsetAsync(ctx->g_vis.p, 0, visw * 4, st));
+        if (nrd > 0) {
+            k_g_build<<<blocks(nrd * nseg, 256), 256, 0, st>>>(
+                act, n_act, d_list, gs, P<int64_t>(E.eoff), P<int64_t>(ctx->g_rdoff), P<int64_t>(ctx->g_capoff), nseg,
+                P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), E.SW,
+                P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt), d_gst + 3);
+            CKL();
+        }
+        if (total > 0) {
+            k_g_graph<<<blocks(total, 256), 256, 0, st>>>(act, n_act, d_list, gs, P<int64_t>(ctx->g_capoff),
+                                                          P<uint64_t>(E.rseq), E.SW, dp, P<uint64_t>(ctx->g_slots),
+                                                          P<uint32_t>(ctx->g_cnt));
+            CKL();
+        }
+        k_g_walk<<<blocks(n_act, 64), 64, 0, st>>>(
+            act, n_act, d_list, gs, P<int64_t>(ctx->g_capoff), P<uint64_t>(E.rseq), E.SW, P<uint64_t>(E.tail),
+            P<uint64_t>(E.tailN), P<int32_t>(E.clen), dp, P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt),
+            P<uint32_t>(ctx->g_vis), P<uint8_t>(ctx->g_cur), P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+            P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), P<int32_t>(ctx->g_still),
+            d_gst + 4);
+        CKL();
+        CK(cudaMemsetAsync(d_ctr, 0, 4, st));
+        k_g_compact<<<blocks(n_act, 256), 256, 0, st>>>(act, n_act, P<int32_t>(ctx->g_still), P<int32_t>(ctx->g_act2), d_ctr);
+        CKL();
+        CK(cudaMemcpyAsync(h, d_ctr, 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        ctx->g_attempts += n_act;
+        n_act = *(int *)h;
+        std::swap(ctx->g_act, ctx->g_act2);
+    }
+    return LA_OK;
+}
+
+la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
+    if (!ctx || !out) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
+    if (!ctx->loaded) return fail(ctx, LA_ERR_STATE, "la_extend before a successful la_load_batch");
+    cudaSetDevice(ctx->device);
+    cudaStream_t st = ctx->stream;
+    Encoded &E = ctx->enc;
+    const DevParams &dp = ctx->dp;
+    const int64_t nE = E.n_ends;
+    const int W = std::max(dp.W, 1);
+    ctx->stats = la_stats{};
+    ctx->g_attempts = 0;
+    ctx->stats.smem_bytes_per_cta = ctx->smem_bytes;
+    ctx->stats.smem_ctas_per_sm = ctx->smem_ctas_per_sm;
+
+    CK(grow(ctx->cls, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->out_len, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->out_term, std::max<int64_t>(nE, 1)));
+    CK(grow(ctx->out_k, std::max<int64_t>(nE, 1)));
+    CK(grow(ctx->out_att, std::max<int64_t>(nE, 1)));
+    CK(grow(ctx->walk_buf, std::max<int64_t>(nE, 1) * W));
+    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->smem_list2, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
+    CK(grow(ctx->ctrs, 256));
+    CK(grow(ctx->gstats, 64));
+    CK(grow(ctx->ext_off, (nE + 1) * 8));
+    CK(grow_host(ctx->h_small, 256));
+    int *d_ctr = P<int>(ctx->ctrs);   // [0]=n_smem [1]=n_glob [2]=work [3]=n_ovf
+    unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
+
+    CK(cudaEventRecord(ctx->ev[0], st));
+    CK(cudaMemsetAsync(d_ctr, 0, 64, st));
+    CK(cudaMemsetAsync(d_gst, 0, 64, st));
+    int *h = (int *)ctx->h_small.p;
+    int n_smem = 0, n_glob = 0;
+    if (nE) {
+        // tuning / test hooks: predicted distinct-kmer fraction used for routing; force the global path
+        const float pred = getenv("LA_PRED_DISTINCT") ? (float)atof(getenv("LA_PRED_DISTINCT")) : 0.5f;
+        const bool force_global = getenv("LA_FORCE_GLOBAL") && atoi(getenv("LA_FORCE_GLOBAL")) != 0;
+        k_plan<<<blocks(nE, 256), 256, 0, st>>>(
+            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW,
+            force_global ? 0u : ctx->smem_bytes, pred,
+            P<int32_t>(ctx->cls), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
+            P<uint8_t>(ctx->out_att), P<int32_t>(ctx->smem_list), P<uint32_t>(ctx->smem_key), d_ctr + 0,
+            P<int32_t>(ctx->glob_list), d_ctr + 1, d_ctr + 4);
+        CKL();
+        CK(cudaMemcpyAsync(h, d_ctr, 24, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        n_smem = h[0];
+        n_glob = h[1];
+        ctx->stats.ends_by_class[0] = h[4];
+        ctx->stats.ends_by_class[1] = h[5];
+    }
+    // LPT order for the persistent kernel: largest expected work first
+    if (n_smem > 1) {
+        size_t tb = 0;
+        cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, P<uint32_t>(ctx->smem_key), P<uint32_t>(ctx->smem_key2),
+                                                  P<int32_t>(ctx->smem_list), P<int32_t>(ctx->smem_list2), n_smem, 0, 32, st);
+        CK(grow(ctx->cub_tmp, tb));
+        cub::DeviceRadixSort::SortPairsDescending(ctx->cub_tmp.p, tb, P<uint32_t>(ctx->smem_key), P<uint32_t>(ctx->smem_key2),
+                                                  P<int32_t>(ctx->smem_list), P<int32_t>(ctx->smem_list2), n_smem, 0, 32, st);
+        CKL();
+        std::swap(ctx->smem_list, ctx->smem_list2);
+    }
+    CK(cudaEventRecord(ctx->ev[1], st));
+    int n_ovf = 0;
+    if (n_smem > 0) {
+        int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
+        const int grid = std::min<int64_t>((int64_t)ctx->n_sm * ctx->smem_ctas_per_sm, n_smem);
+        k_smem<256><<<grid, 256, ctx->smem_bytes, st>>>(
+            P<int32_t>(ctx->smem_list), n_smem, d_ctr + 2, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
+            P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
+            P<int32_t>(E.clen), E.SW, dp, ctx->smem_bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+            P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 3,
+            (GlobalStats *)d_gst);
+        CKL();
+        CK(cudaMemcpyAsync(h, d_ctr + 3, 4, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        n_ovf = h[0];
+        if (n_ovf) {   // append the overflowed ends to the global list
+            CK(cudaMemcpyAsync(P<int32_t>(ctx->glob_list) + n_glob, ovf_list, (size_t)n_ovf * 4,
+                               cudaMemcpyDeviceToDevice, st));
+        }
+    }
+    CK(cudaEventRecord(ctx->ev[2], st));
+    la_status s = run_global(ctx, P<int32_t>(ctx->glob_list), n_glob + n_ovf, nullptr);
+    if (s != LA_OK) return s;
+    CK(cudaEventRecord(ctx->ev[3], st));
+    // emit: exclusive scan of lengths -> ext_off; compact + reverse-complement LEFT ends
+    {
+        CK(grow(ctx->lens64, (nE + 1) * 8));
+        k_len64<<<blocks(nE + 1, 256), 256, 0, st>>>(P<int32_t>(ctx->out_len), nE, P<int64_t>(ctx->lens64));
+        CKL();
+        size_t tb = 0;
+        cub::DeviceScan::ExclusiveSum(nullptr, tb, P<int64_t>(ctx->lens64), P<int64_t>(ctx->ext_off), nE + 1, st);
+        CK(grow(ctx->cub_tmp, tb));
+        cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->lens64), P<int64_t>(ctx->ext_off), nE + 1, st);
+        CKL();
+    }
+    int64_t *h64 = (int64_t *)ctx->h_small.p;
+    CK(cudaMemcpyAsync(h64, P<int64_t>(ctx->ext_off) + nE, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64 + 1, d_gst, 40, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const int64_t total = h64[0];
+    // d_gst: [0] smem inserts [1] smem walk steps [2] smem attempts [3] global inserts [4] global steps
+    ctx->stats.inserts = h64[1] + h64[4];
+    ctx->stats.inserts_smem = h64[1];
+    ctx->stats.walk_steps = h64[2] + h64[5];
+    ctx->stats.attempts = h64[3] + ctx->g_attempts;
+    ctx->stats.ext_bases = total;
+    CK(grow(ctx->ext_seq, total + 16));
+    if (nE) {
+        k_emit<<<blocks(nE * 32, 256), 256, 0, st>>>(P<uint8_t>(ctx->walk_buf), W, P<int64_t>(ctx->ext_off), nE,
+                                                     P<char>(ctx->ext_seq));
+        CKL();
+    }
+    CK(cudaEventRecord(ctx->ev[4], st));
+    if (to_host) {
+        CK(grow_host(ctx->h_ext_off, (nE + 1) * 8));
+        CK(grow_host(ctx->h_ext_seq, total + 16));
+        CK(grow_host(ctx->h_term, nE + 16));
+        CK(grow_host(ctx->h_k, nE + 16));
+        CK(grow_host(ctx->h_att, nE + 16));
+        CK(cudaMemcpyAsync(ctx->h_ext_off.p, ctx->ext_off.p, (nE + 1) * 8, cudaMemcpyDeviceToHost, st));
+        if (total) CK(cudaMemcpyAsync(ctx->h_ext_seq.p, ctx->ext_seq.p, total, cudaMemcpyDeviceToHost, st));
+        if (nE) {
+            CK(cudaMemcpyAsync(ctx->h_term.p, ctx->out_term.p, nE, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(ctx->h_k.p, ctx->out_k.p, nE, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync(ctx->h_att.p, ctx->out_att.p, nE, cudaMemcpyDeviceToHost, st));
+        }
+        out->ext_off = (const int64_t *)ctx->h_ext_off.p;
+        out->ext_seq = (const char *)ctx->h_ext_seq.p;
+        out->term = (const uint8_t *)ctx->h_term.p;
+        out->k_used = (const uint8_t *)ctx->h_k.p;
+        out->n_attempts = (const uint8_t *)ctx->h_att.p;
+    } else {
+        out->ext_off = P<int64_t>(ctx->ext_off);
+        out->ext_seq = P<char>(ctx->ext_seq);
+        out->term = P<uint8_t>(ctx->out_term);
+        out->k_used = P<uint8_t>(ctx->out_k);
+        out->n_attempts = P<uint8_t>(ctx->out_att);
+    }
+    out->n_ends = nE;
+    CK(cudaStreamSynchronize(st));
+    float ms = 0;
+    cudaEventElapsedTime(&ms, ctx->ev[0], ctx->ev[4]);
+    ctx->stats.ms_total = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[2]);
+    ctx->stats.ms_smem = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[2], ctx->ev[3]);
+    ctx->stats.ms_global = ms;
+    cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
+    ctx->stats.ms_emit = ms;
+    // class counts (host-side tally from the plan counters)
+    ctx->stats.ends_by_class[2] = n_smem - n_ovf;
+    ctx->stats.ends_by_class[3] = n_glob;
+    ctx->stats.ends_by_class[4] = n_ovf;
+    return LA_OK;
+}
+
+}  // namespace
+
+extern "C" la_status la_extend(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, true); }
+extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, false); }

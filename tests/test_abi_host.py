@@ -1,0 +1,59 @@
+"""Host-side checks of the C-ABI library (no GPU): it loads, exports every symbol include/locassm.h
+declares, and its host helpers follow the paper's sizing rule."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_sc_awanhedbdoy21_b200 import build, _lib
+    build.build()
+    return _lib.load()
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "locassm.h")).read()
+    return sorted(set(re.findall(r"^\s*(?:la_status|const char \*|int64_t|double)\s*\*?\s*(la_\w+)\s*\(", src, re.M)))
+
+
+def test_exports_every_declared_symbol(lib):
+    names = declared_symbols()
+    assert set(names) >= {"la_create", "la_load_batch", "la_extend", "la_destroy"}
+    for n in names:
+        assert hasattr(lib, n), n
+
+
+def test_load_factor_helper(lib):
+    """P1: table size l*r for (l-k+1)*r k-mers -> load factor (l-k+1)/l; 0.93 at (300, 21)."""
+    assert abs(lib.la_paper_load_factor(300, 21) - 280 / 300) < 1e-12
+    assert round(lib.la_paper_load_factor(300, 21), 2) == 0.93
+
+
+def test_global_capacity_bound(lib):
+    """The global-table capacity keeps the load factor <= 0.7 even if every insert is distinct."""
+    for n in (0, 1, 117, 5000, 10 ** 6, 5 * 10 ** 7):
+        cap = lib.la_plan_global_capacity(n)
+        assert cap >= n + 1 and n <= 0.7 * cap + 1e-9
+
+
+def test_no_gpu_create_fails_cleanly(lib):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    c = ctypes.c_void_p()
+    assert lib.la_create(ctypes.byref(c), 0, None) == -3
+    assert lib.la_destroy(None) == 0
+
+
+def test_product_never_imports_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_sc_awanhedbdoy21_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "oracle" not in re.sub(r"#.*|//.*", "", txt).replace("oracle/", ""), f

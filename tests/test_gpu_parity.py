@@ -1,0 +1,196 @@
+"""GPU parity: the CUDA library (through the C ABI) against the CPU oracle, end by end, bit-exact
+(extension string, termination code, k of the returned walk, attempts) — DESIGN.md §5.
+
+All inputs are seeded and synthetic (gen/); expected values come only from oracle/ or from closed
+forms of the constructions.
+"""
+import os
+
+import numpy as np
+import pytest
+
+from conftest import cached_batch
+from gen import Params
+from gen import cases as C
+
+pytestmark = pytest.mark.gpu
+
+P0 = Params()
+
+
+@pytest.fixture(scope="module")
+def LA():
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    la = LocalAssembler(0)
+    yield la
+    la.close()
+
+
+def check(LA, orc, batch, P, ends=None, env=None):
+    old = {}
+    for k, v in (env or {}).items():
+        old[k] = os.environ.get(k)
+        os.environ[k] = v
+    try:
+        r = LA.load(batch, P).extend()
+        st = LA.stats()
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    ref = orc.extend(batch, P, ends=ends)
+    sel = ref["ends"]
+    got = r.ext_list()
+    bad = [int(e) for i, e in enumerate(sel) if got[e] != ref["ext"][i]
+           or r.term[e] != ref["term"][i] or r.k_used[e] != ref["k_used"][i]
+           or r.n_attempts[e] != ref["n_attempts"][i]]
+    if bad:
+        e = bad[0]
+        i = int(np.nonzero(sel == e)[0][0])
+        raise AssertionError(
+            f"{len(bad)}/{len(sel)} ends differ; first end {e}: gpu=({got[e][:40]}..., len {len(got[e])}, "
+            f"term {r.term[e]}, k {r.k_used[e]}, att {r.n_attempts[e]}) oracle=({ref['ext'][i][:40]}..., len "
+            f"{len(ref['ext'][i])}, term {ref['term'][i]}, k {ref['k_used'][i]}, att {ref['n_attempts'][i]})")
+    if ends is None:
+        assert st["inserts"] == int(ref["inserts"].sum())
+        assert st["walk_steps"] == int(ref["walk_steps"].sum())
+        assert st["ext_bases"] == sum(len(x) for x in ref["ext"])
+    return r, st
+
+
+def test_c1_single_k(LA, orc):
+    check(LA, orc, cached_batch("C1"), Params(k_start=21, k_min=21, k_max=21))
+
+
+def test_c2_small_full_schedule(LA, orc):
+    r, st = check(LA, orc, cached_batch("C2", scale=0.03), P0)
+    assert st["ends_by_class"][2] > 0
+
+
+def test_c2_small_forced_global(LA, orc):
+    _, st = check(LA, orc, cached_batch("C2", scale=0.03), P0, env={"LA_FORCE_GLOBAL": "1"})
+    assert st["ends_by_class"][2] == 0 and st["ends_by_class"][3] > 0
+
+
+def test_c2_small_forced_overflow(LA, orc):
+    """Route everything to shared memory: ends whose tables overflow are redone in global memory."""
+    _, st = check(LA, orc, cached_batch("C2", scale=0.03), P0, env={"LA_PRED_DISTINCT": "0.01"})
+    assert st["ends_by_class"][4] > 0
+
+
+@pytest.mark.parametrize("P", [
+    Params(k_start=25, k_min=17, k_max=45, k_shift=4, max_walk_len=120, q_lo=5, q_hi=30, min_votes=3,
+           min_frac_pct=30),
+    Params(k_start=31, k_min=31, k_max=128, k_shift=16, min_votes=1, min_frac_pct=0),
+    Params(k_start=64, k_min=32, k_max=96, k_shift=32, max_walk_len=1024),
+    Params(k_start=9, k_min=5, k_max=13, k_shift=2, max_walk_len=50),
+    Params(max_walk_len=0),
+])
+def test_c2_small_params(LA, orc, P):
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(300))
+    check(LA, orc, b, P)
+
+
+def test_c3_sampled(LA, orc):
+    """High-skew workload: every hot end (global path) and a sample of sparse ends."""
+    b = cached_batch("C3")
+    r = b.reads_per_end()
+    hot = np.nonzero(r >= 10000)[0][:3]
+    rng = np.random.default_rng(0)
+    ends = np.concatenate([hot, rng.choice(b.n_ends, 300, replace=False)])
+    _, st = check(LA, orc, b, P0, ends=ends)
+    assert st["ends_by_class"][3] >= len(hot)
+
+
+def test_pins_on_gpu(LA, orc):
+    """Closed-form constructions (P2-P8) through the GPU path, batched as one multi-contig batch."""
+    rng = np.random.default_rng(1)
+    G = C.unique_genome(rng, 1200)
+    contigs, ends = [], []
+    # P2 DEADEND chain, P6 MAXLEN, P7 N in contig, P8 NOREADS/SHORT/short reads
+    for e, a_hi in ((500, 600), (500, 1000)):
+        contigs.append(G[e - 200:e]); ends += [C.tile(G, 0, 250, 150, qchar="5"), C.tile(G, 200, a_hi, 150)]
+    nc = list(G[300:500]); nc[200 - 1 - 27] = "N"
+    contigs.append("".join(nc)); ends += [[], C.tile(G, 200, 600, 150)]
+    contigs.append(G[468:500]); ends += [[], C.tile(G, 200, 600, 150)]
+    contigs.append(G[300:500]); ends += [[], [(s[:21], q[:21]) for s, q in C.tile(G, 200, 600, 150)]]
+    u = 110
+    while True:
+        U, FL, FR = C.random_seq(rng, u), C.random_seq(rng, 200), C.random_seq(rng, 200)
+        if C.kmers_unique(FL + U + FR, 21):
+            break
+    reg = FL + U * 7 + FR
+    contigs.append(reg[300:580]); ends += [[], C.tile(reg, 0, len(reg) - 150, 150)]
+    b = C.Batch.from_lists(contigs, ends)
+    r, _ = check(LA, orc, b, P0)
+    assert r.ext(1) == G[500:749] and r.term[1] == 0
+    assert r.ext(3) == G[500:800] and r.term[3] == 3
+    assert r.k_used[5] == 25
+    assert r.term[6] == 4 and r.term[7] == 5
+    assert r.ext(9) == "" and r.term[9] == 0
+    assert r.ext(11) == reg[580:690] and r.term[11] == 2
+
+
+def test_rc_twin_and_permutation(LA, orc):
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(200))
+    r = LA.load(b, P0).extend()
+    ext = r.ext_list()
+    tw = C.twin(b)
+    rt = LA.load(tw, P0).extend()
+    ext_t = rt.ext_list()
+    for c in range(b.n_contigs):
+        assert ext_t[2 * c] == C.rc(ext[2 * c + 1]) and ext_t[2 * c + 1] == C.rc(ext[2 * c])
+    bp, perm = C.permuted(b, 5)
+    rp = LA.load(bp, P0).extend()
+    idx = np.stack([2 * perm, 2 * perm + 1], 1).reshape(-1)
+    assert [ext[i] for i in idx] == rp.ext_list()
+    assert np.array_equal(r.term[idx], rp.term)
+
+
+def test_device_memory_input(LA, orc):
+    import torch
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(150))
+    host = LA.load(b, P0).extend()
+
+    class DevBatch:
+        pass
+    d = DevBatch()
+    for f in ("contig_seq", "contig_off", "read_seq", "read_qual", "read_off", "end_read_off"):
+        setattr(d, f, torch.from_numpy(getattr(b, f)).cuda())
+    dev = LA.load(d, P0).extend()
+    assert host.ext_list() == dev.ext_list() and np.array_equal(host.term, dev.term)
+
+
+def test_empty_and_degenerate(LA, orc):
+    check(LA, orc, C.Batch.from_lists([], []), P0)
+    check(LA, orc, C.Batch.from_lists(["ACGT" * 10, "A"], [[], [], [], []]), P0)
+    # reads of length 0 and reads of only N
+    check(LA, orc, C.Batch.from_lists(["ACGT" * 20], [[("", "")], [("N" * 150, "I" * 150)]]), P0)
+
+
+def test_invalid_inputs_leave_context_unchanged(LA, orc):
+    from paper_conf_sc_awanhedbdoy21_b200._lib import LocAssmError
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(50))
+    good = LA.load(b, P0).extend().ext_list()
+    bad = C.Batch.from_lists(["ACGTX" * 10], [[], []])
+    with pytest.raises(LocAssmError, match="INVALID_ARG"):
+        LA.load(bad, P0)
+    bad2 = C.Batch.from_lists(["ACGT" * 10], [[], [("A" * 301, "I" * 301)]])
+    with pytest.raises(LocAssmError, match="300"):
+        LA.load(bad2, P0)
+    bad3 = C.Batch.from_lists(["ACGT" * 10], [[], [("ACGT", "I!II")]])
+    with pytest.raises(LocAssmError, match="qual"):
+        LA.load(bad3, P0.replace(qual_offset=40))
+    with pytest.raises(LocAssmError, match="k schedule"):
+        LA.load(b, P0.replace(k_start=10))
+    assert LA.extend().ext_list() == good
+
+
+def test_state_error_before_load():
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    from paper_conf_sc_awanhedbdoy21_b200._lib import LocAssmError
+    with LocalAssembler(0) as la:
+        with pytest.raises(LocAssmError, match="STATE"):
+            la.extend()
