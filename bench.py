@@ -131,8 +131,8 @@ def roofline_peaks():
         peaks["hbm_src"] = "fallback (B200_PROFILING.md)"
     try:
         m = json.load(open(os.path.join(ROOT, "profiles", "micro_random_update.json")))
-        peaks["smem_gups"] = m["smem_atomic_add"]
-        peaks["smem_src"] = "profiles/micro_random_update.json (smem_atomic_add, measured on B200)"
+        peaks["smem_gups"] = m["smem_atomic_add32"]
+        peaks["smem_src"] = "profiles/micro_random_update.json (smem_atomic_add32, measured on B200)"
     except Exception:
         peaks["smem_gups"] = None
         peaks["smem_src"] = "unmeasured"

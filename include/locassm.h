@@ -104,9 +104,11 @@ typedef struct {
     int64_t ext_bases;        /* total extension length                                          */
     int64_t ends_by_class[5]; /* NOREADS, SHORT, SMEM, GLOBAL, SMEM->GLOBAL (smem table overflow) */
     int64_t kernel_launches;  /* kernels launched by the last la_extend                          */
-    int64_t smem_bytes_per_cta;
+    int64_t smem_bytes_per_cta;  /* small-table kernel                                          */
     int32_t smem_ctas_per_sm;
     int32_t global_rounds;
+    int64_t ends_medium;         /* ends routed to the medium (one CTA per SM) kernel             */
+    double ms_smem_medium;       /* its device time (included in ms_smem)                          */
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);

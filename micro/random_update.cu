@@ -1,6 +1,8 @@
 // random_update.cu — microbenchmarks of the roofline denominators:
 // the random-update rate of the memory that holds a k-mer table.
-//   smem_atomic_add : random 32-bit atomicAdd into a per-CTA shared-memory table (ATOMS.ADD)
+//   smem_atomic_inc32: random 32-bit atomicAdd(+1) into a per-CTA shared-memory table (ATOMS.POPC.INC)
+//   smem_atomic_add32: random 32-bit atomicAdd of a variable increment, old value returned (ATOMS.ADD)
+//                      = the vote update of the table
 //   smem_cas64      : random 64-bit atomicCAS into shared memory (ATOMS.CAS.64)
 //   smem_load64     : random 64-bit loads from shared memory (LDS.64, the probe)
 //   global_red_l2   : random 32-bit atomicAdd (RED.ADD) into a 64 MB L2-resident global table
@@ -27,6 +29,8 @@ __global__ void k_smem(int iters, uint32_t words, unsigned long long *sink) {
         x = hsh(x + it);
         if (MODE == 0) {
             atomicAdd(&t[x % words], 1u);
+        } else if (MODE == 3) {   // the table's vote update: 32-bit add of a data-dependent increment
+            acc += atomicAdd(&t[x % words], 1u << ((x >> 24) & 31));
         } else if (MODE == 1) {
             unsigned long long *t64 = (unsigned long long *)t;
             acc += atomicCAS(&t64[x % (words / 2)], 0ull, (unsigned long long)x);
@@ -61,17 +65,19 @@ int main() {
     const uint32_t bytes = 110 * 1024;
     const uint32_t words = bytes / 4;
     const int iters = 4096;
-    double res[5] = {0, 0, 0, 0, 0};
+    double res[6] = {0, 0, 0, 0, 0, 0};
     cudaFuncSetAttribute(k_smem<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     cudaFuncSetAttribute(k_smem<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     cudaFuncSetAttribute(k_smem<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
-    for (int mode = 0; mode < 3; ++mode) {
+    cudaFuncSetAttribute(k_smem<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    for (int mode = 0; mode < 4; ++mode) {
         double best = 0;
         for (int rep = 0; rep < 6; ++rep) {
             cudaEventRecord(a);
             if (mode == 0) k_smem<0><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
             if (mode == 1) k_smem<1><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
             if (mode == 2) k_smem<2><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
+            if (mode == 3) k_smem<3><<<sms * ctas_per_sm, threads, bytes>>>(iters, words, sink);
             cudaEventRecord(b);
             cudaEventSynchronize(b);
             float ms;
@@ -99,13 +105,13 @@ int main() {
             double ops = (double)grid * 256 * gi;
             if (rep) best = best > ops / ms / 1e6 ? best : ops / ms / 1e6;
         }
-        res[3 + g] = best;
+        res[4 + g] = best;
         cudaFree(tab);
     }
-    printf("{\"unit\": \"G updates/s\", \"smem_atomic_add\": %.2f, \"smem_cas64\": %.2f, \"smem_load64\": %.2f, "
-           "\"global_red_l2\": %.2f, \"global_red_hbm\": %.2f, \"sms\": %d, \"smem_ctas_per_sm\": %d, "
-           "\"threads\": %d, \"smem_bytes_per_cta\": %u, \"err\": \"%s\"}\n",
-           res[0], res[1], res[2], res[3], res[4], sms, ctas_per_sm, threads, bytes,
+    printf("{\"unit\": \"G updates/s\", \"smem_atomic_inc32\": %.2f, \"smem_cas64\": %.2f, \"smem_load64\": %.2f, "
+           "\"smem_atomic_add32\": %.2f, \"global_red_l2\": %.2f, \"global_red_hbm\": %.2f, \"sms\": %d, "
+           "\"smem_ctas_per_sm\": %d, \"threads\": %d, \"smem_bytes_per_cta\": %u, \"err\": \"%s\"}\n",
+           res[0], res[1], res[2], res[3], res[4], res[5], sms, ctas_per_sm, threads, bytes,
            cudaGetErrorString(cudaGetLastError()));
     return 0;
 }

@@ -45,7 +45,8 @@ class la_stats(ctypes.Structure):
                 ("attempts", ctypes.c_int64), ("ext_bases", ctypes.c_int64),
                 ("ends_by_class", ctypes.c_int64 * 5), ("kernel_launches", ctypes.c_int64),
                 ("smem_bytes_per_cta", ctypes.c_int64), ("smem_ctas_per_sm", ctypes.c_int32),
-                ("global_rounds", ctypes.c_int32)]
+                ("global_rounds", ctypes.c_int32), ("ends_medium", ctypes.c_int64),
+                ("ms_smem_medium", ctypes.c_double)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_get_stats",

@@ -4,6 +4,7 @@ nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -shared -Xcompiler -f
 """
 from __future__ import annotations
 
+import glob
 import os
 import subprocess
 import sys
@@ -12,8 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SO = os.path.join(HERE, "liblocassm.so")
 SRC = [os.path.join(HERE, "csrc", "locassm.cu")]
-DEPS = SRC + [os.path.join(HERE, "csrc", f) for f in ("la_device.cuh", "la_kernels.cuh")] + \
-    [os.path.join(ROOT, "include", "locassm.h")]
+DEPS = SRC + sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu*"))) + [os.path.join(ROOT, "include", "locassm.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-shared", "-Xcompiler", "-fPIC", "-I" + os.path.join(ROOT, "include")]

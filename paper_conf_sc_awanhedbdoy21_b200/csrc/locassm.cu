@@ -61,8 +61,8 @@ struct la_ctx {
     bool loaded = false;
     std::string err;
     int n_sm = 148;
-    int smem_ctas_per_sm = 2;
-    uint32_t smem_bytes = 0;
+    int ctas_S = 3;               // small-table CTAs per SM
+    uint32_t bytes_S = 0, bytes_M = 0;   // dynamic shared memory per CTA: small / medium kernel
     la_params params{};
     DevParams dp{};
     Encoded enc, spare;   // current encoding; la_load_batch fills `spare` and swaps on success
@@ -173,11 +173,12 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     cudaDeviceProp prop;
     cudaGetDeviceProperties(&prop, device);
     ctx->n_sm = prop.multiProcessorCount;
-    if (const char *s = getenv("LA_SMEM_CTAS")) ctx->smem_ctas_per_sm = std::max(1, atoi(s));
+    if (const char *s = getenv("LA_SMEM_CTAS")) ctx->ctas_S = std::max(1, atoi(s));
     // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
-    size_t per = prop.sharedMemPerMultiprocessor / ctx->smem_ctas_per_sm - 1024 - 512 /* static */;
-    per = std::min(per, (size_t)prop.sharedMemPerBlockOptin);
-    ctx->smem_bytes = (uint32_t)(per & ~(size_t)127);
+    size_t per = prop.sharedMemPerMultiprocessor / ctx->ctas_S - 1024 - 512 /* static */;
+    per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - 512);
+    ctx->bytes_S = (uint32_t)(per & ~(size_t)127);
+    ctx->bytes_M = (uint32_t)((prop.sharedMemPerBlockOptin - 512) & ~(size_t)127);
     if (cuda_stream) ctx->stream = (cudaStream_t)cuda_stream;
     else {
         if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) {
@@ -187,8 +188,8 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
-    if (cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->smem_bytes) !=
-        cudaSuccess) {
+    if (cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->bytes_S) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->bytes_M) != cudaSuccess) {
         cudaGetLastError();
         la_destroy(ctx);
         return LA_ERR_CUDA;
@@ -398,55 +399,67 @@ la_status run_global(la_ctx *ctx, const int32_t *d_list, int n_list, double *ms_
     int n_act = n_list;
     const int nseg = std::max(1, (E.maxlen - dp.k_min + GSEG - 1) / GSEG);   // positions per read
     int64_t *h = (int64_t *)ctx->h_small.p;
+    // memory budget of one wave of global tables (slots: 8 B key + 32 B counters + 1 visited bit)
+    const int64_t budget = (getenv("LA_GLOBAL_BUDGET_MB") ? atoll(getenv("LA_GLOBAL_BUDGET_MB")) : 8192) << 20;
+    std::vector<int64_t> hcap, hnrd, capoff, rdoff;
     while (n_act > 0) {
         ctx->stats.global_rounds++;
         int32_t *act = P<int32_t>(ctx->g_act);
         k_g_caps<<<n_act, 256, 0, st>>>(act, n_act, d_list, gs, P<int64_t>(E.eoff), P<uint16_t>(E.rlen),
                                         P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_nrd));
         CKL();
-        size_t tb = 0;
-        cub::DeviceScan::ExclusiveSum(nullptr, tb, P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_capoff), n_act + 1, st);
-        CK(grow(ctx->cub_tmp, tb));
-        // the element past the end is 0 -> offsets[n] = total
-        CK(cudaMemsetAsync(P<int64_t>(ctx->g_cap) + n_act, 0, 8, st));
-        CK(cudaMemsetAsync(P<int64_t>(ctx->g_nrd) + n_act, 0, 8, st));
-        CK(cudaGetLastError());
-        cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->g_cap), P<int64_t>(ctx->g_capoff), n_act + 1, st);
-        CKL();
-        cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->g_nrd), P<int64_t>(ctx->g_rdoff), n_act + 1, st);
-        CKL();
-        CK(cudaMemcpyAsync(h, P<int64_t>(ctx->g_capoff) + n_act, 8, cudaMemcpyDeviceToHost, st));
-        CK(cudaMemcpyAsync(h + 1, P<int64_t>(ctx->g_rdoff) + n_act, 8, cudaMemcpyDeviceToHost, st));
+        hcap.resize(n_act);
+        hnrd.resize(n_act);
+        CK(cudaMemcpyAsync(hcap.data(), ctx->g_cap.p, (size_t)n_act * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(hnrd.data(), ctx->g_nrd.p, (size_t)n_act * 8, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
-        const int64_t total = h[0], nrd = h[1];
-        if (total >= (int64_t)NONE) return fail(ctx, LA_ERR_CAPACITY, "global table round too large (%lld slots)", (long long)total);
-        CK(grow(ctx->g_slots, (size_t)total * 8));
-        CK(grow(ctx->g_cnt, (size_t)total * 32));
-        const size_t visw = (size_t)(total >> 5) + n_act + 2;
-        CK(grow(ctx->g_vis, visw * 4));
-        CK(cudaMemsetAsync(ctx->g_slots.p, 0, (size_t)total * 8, st));
-        CK(cudaMemsetAsync(ctx->g_cnt.p, 0, (size_t)total * 32, st));
-        CK(cudaMemsetAsync(ctx->g_vis.p, 0, visw * 4, st));
-        if (nrd > 0) {
-            k_g_build<<<blocks(nrd * nseg, 256), 256, 0, st>>>(
-                act, n_act, d_list, gs, P<int64_t>(E.eoff), P<int64_t>(ctx->g_rdoff), P<int64_t>(ctx->g_capoff), nseg,
-                P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), E.SW,
-                P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt), d_gst + 3);
+        // waves of consecutive active ends whose tables fit the budget
+        for (int a = 0; a < n_act;) {
+            int b = a;
+            int64_t tot = 0, nrd = 0;
+            capoff.assign(1, 0);
+            rdoff.assign(1, 0);
+            while (b < n_act && (b == a || (tot + hcap[b]) * 41 <= budget)) {
+                if (hcap[b] >= (int64_t)NONE)
+                    return fail(ctx, LA_ERR_CAPACITY, "global table of one end too large (%lld slots)", (long long)hcap[b]);
+                tot += hcap[b];
+                nrd += hnrd[b];
+                capoff.push_back(tot);
+                rdoff.push_back(nrd);
+                ++b;
+            }
+            const int n = b - a;
+            CK(cudaMemcpyAsync(ctx->g_capoff.p, capoff.data(), (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, st));
+            CK(cudaMemcpyAsync(ctx->g_rdoff.p, rdoff.data(), (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, st));
+            CK(grow(ctx->g_slots, (size_t)tot * 8));
+            CK(grow(ctx->g_cnt, (size_t)tot * 32));
+            const size_t visw = (size_t)(tot >> 5) + n + 2;
+            CK(grow(ctx->g_vis, visw * 4));
+            CK(cudaMemsetAsync(ctx->g_slots.p, 0, (size_t)tot * 8, st));
+            CK(cudaMemsetAsync(ctx->g_cnt.p, 0, (size_t)tot * 32, st));
+            CK(cudaMemsetAsync(ctx->g_vis.p, 0, visw * 4, st));
+            if (nrd > 0) {
+                k_g_build<<<blocks(nrd * nseg, 256), 256, 0, st>>>(
+                    act + a, n, d_list, gs, P<int64_t>(E.eoff), P<int64_t>(ctx->g_rdoff), P<int64_t>(ctx->g_capoff),
+                    nseg, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), E.SW,
+                    P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt), d_gst + 3);
+                CKL();
+            }
+            if (tot > 0) {
+                k_g_graph<<<blocks(tot, 256), 256, 0, st>>>(act + a, n, d_list, gs, P<int64_t>(ctx->g_capoff),
+                                                            P<uint64_t>(E.rseq), E.SW, dp, P<uint64_t>(ctx->g_slots),
+                                                            P<uint32_t>(ctx->g_cnt));
+                CKL();
+            }
+            k_g_walk<<<blocks(n, 64), 64, 0, st>>>(
+                act + a, n, d_list, gs, P<int64_t>(ctx->g_capoff), P<uint64_t>(E.rseq), E.SW, P<uint64_t>(E.tail),
+                P<uint64_t>(E.tailN), P<int32_t>(E.clen), dp, P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt),
+                P<uint32_t>(ctx->g_vis), P<uint8_t>(ctx->g_cur), P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+                P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
+                P<int32_t>(ctx->g_still) + a, d_gst + 4);
             CKL();
+            a = b;
         }
-        if (total > 0) {
-            k_g_graph<<<blocks(total, 256), 256, 0, st>>>(act, n_act, d_list, gs, P<int64_t>(ctx->g_capoff),
-                                                          P<uint64_t>(E.rseq), E.SW, dp, P<uint64_t>(ctx->g_slots),
-                                                          P<uint32_t>(ctx->g_cnt));
-            CKL();
-        }
-        k_g_walk<<<blocks(n_act, 64), 64, 0, st>>>(
-            act, n_act, d_list, gs, P<int64_t>(ctx->g_capoff), P<uint64_t>(E.rseq), E.SW, P<uint64_t>(E.tail),
-            P<uint64_t>(E.tailN), P<int32_t>(E.clen), dp, P<uint64_t>(ctx->g_slots), P<uint32_t>(ctx->g_cnt),
-            P<uint32_t>(ctx->g_vis), P<uint8_t>(ctx->g_cur), P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
-            P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), P<int32_t>(ctx->g_still),
-            d_gst + 4);
-        CKL();
         CK(cudaMemsetAsync(d_ctr, 0, 4, st));
         k_g_compact<<<blocks(n_act, 256), 256, 0, st>>>(act, n_act, P<int32_t>(ctx->g_still), P<int32_t>(ctx->g_act2), d_ctr);
         CKL();
@@ -471,8 +484,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     const int W = std::max(dp.W, 1);
     ctx->stats = la_stats{};
     ctx->g_attempts = 0;
-    ctx->stats.smem_bytes_per_cta = ctx->smem_bytes;
-    ctx->stats.smem_ctas_per_sm = ctx->smem_ctas_per_sm;
+    ctx->stats.smem_bytes_per_cta = ctx->bytes_S;
+    ctx->stats.smem_ctas_per_sm = ctx->ctas_S;
 
     CK(grow(ctx->cls, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->out_len, std::max<int64_t>(nE, 1) * 4));
@@ -480,8 +493,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->out_k, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->out_att, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->walk_buf, std::max<int64_t>(nE, 1) * W));
-    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4));
-    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4));
+    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 8));
+    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 8));
     CK(grow(ctx->smem_list2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
@@ -489,62 +502,81 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->gstats, 64));
     CK(grow(ctx->ext_off, (nE + 1) * 8));
     CK(grow_host(ctx->h_small, 256));
-    int *d_ctr = P<int>(ctx->ctrs);   // [0]=n_smem [1]=n_glob [2]=work [3]=n_ovf
+    int *d_ctr = P<int>(ctx->ctrs);   // [0] n_S [1] n_M [2] n_G [3] NOREADS [4] SHORT [5,6] work [7] n_ovf
     unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
 
     CK(cudaEventRecord(ctx->ev[0], st));
     CK(cudaMemsetAsync(d_ctr, 0, 64, st));
     CK(cudaMemsetAsync(d_gst, 0, 64, st));
     int *h = (int *)ctx->h_small.p;
-    int n_smem = 0, n_glob = 0;
+    int n_S = 0, n_M = 0, n_glob = 0;
+    int32_t *list_S = P<int32_t>(ctx->smem_list), *list_M = P<int32_t>(ctx->smem_list) + nE;
+    uint32_t *key_S = P<uint32_t>(ctx->smem_key), *key_M = P<uint32_t>(ctx->smem_key) + nE;
     if (nE) {
-        // tuning / test hooks: predicted distinct-kmer fraction used for routing; force the global path
-        const float pred = getenv("LA_PRED_DISTINCT") ? (float)atof(getenv("LA_PRED_DISTINCT")) : 0.5f;
+        // test hook: force every end with reads onto the global path
         const bool force_global = getenv("LA_FORCE_GLOBAL") && atoi(getenv("LA_FORCE_GLOBAL")) != 0;
+        // test hook: pretend every end fits the small-table kernel (exercises the overflow redo)
+        const bool force_smem = getenv("LA_FORCE_SMEM") && atoi(getenv("LA_FORCE_SMEM")) != 0;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
             P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW,
-            force_global ? 0u : ctx->smem_bytes, pred,
+            force_global ? 0u : (force_smem ? 0xffffffffu : ctx->bytes_S), force_global ? 0u : ctx->bytes_M,
             P<int32_t>(ctx->cls), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), P<int32_t>(ctx->smem_list), P<uint32_t>(ctx->smem_key), d_ctr + 0,
-            P<int32_t>(ctx->glob_list), d_ctr + 1, d_ctr + 4);
+            P<uint8_t>(ctx->out_att), list_S, key_S, list_M, key_M, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
-        CK(cudaMemcpyAsync(h, d_ctr, 24, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h, d_ctr, 20, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
-        n_smem = h[0];
-        n_glob = h[1];
-        ctx->stats.ends_by_class[0] = h[4];
-        ctx->stats.ends_by_class[1] = h[5];
+        n_S = h[0];
+        n_M = h[1];
+        n_glob = h[2];
+        ctx->stats.ends_by_class[0] = h[3];
+        ctx->stats.ends_by_class[1] = h[4];
     }
-    // LPT order for the persistent kernel: largest expected work first
-    if (n_smem > 1) {
+    // LPT order for the persistent kernels: largest expected work first
+    for (int cls = 0; cls < 2; ++cls) {
+        const int n = cls ? n_M : n_S;
+        if (n < 2) continue;
+        int32_t *lst = cls ? list_M : list_S;
+        uint32_t *key = cls ? key_M : key_S;
         size_t tb = 0;
-        cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, P<uint32_t>(ctx->smem_key), P<uint32_t>(ctx->smem_key2),
-                                                  P<int32_t>(ctx->smem_list), P<int32_t>(ctx->smem_list2), n_smem, 0, 32, st);
+        cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, key, P<uint32_t>(ctx->smem_key2), lst,
+                                                  P<int32_t>(ctx->smem_list2), n, 0, 32, st);
         CK(grow(ctx->cub_tmp, tb));
-        cub::DeviceRadixSort::SortPairsDescending(ctx->cub_tmp.p, tb, P<uint32_t>(ctx->smem_key), P<uint32_t>(ctx->smem_key2),
-                                                  P<int32_t>(ctx->smem_list), P<int32_t>(ctx->smem_list2), n_smem, 0, 32, st);
+        cub::DeviceRadixSort::SortPairsDescending(ctx->cub_tmp.p, tb, key, P<uint32_t>(ctx->smem_key2), lst,
+                                                  P<int32_t>(ctx->smem_list2), n, 0, 32, st);
         CKL();
-        std::swap(ctx->smem_list, ctx->smem_list2);
+        CK(cudaMemcpyAsync(lst, ctx->smem_list2.p, (size_t)n * 4, cudaMemcpyDeviceToDevice, st));
     }
     CK(cudaEventRecord(ctx->ev[1], st));
-    int n_ovf = 0;
-    if (n_smem > 0) {
-        int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
-        const int grid = std::min<int64_t>((int64_t)ctx->n_sm * ctx->smem_ctas_per_sm, n_smem);
-        k_smem<256><<<grid, 256, ctx->smem_bytes, st>>>(
-            P<int32_t>(ctx->smem_list), n_smem, d_ctr + 2, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
-            P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
-            P<int32_t>(E.clen), E.SW, dp, ctx->smem_bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
-            P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 3,
-            (GlobalStats *)d_gst);
+    int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
+    // medium ends first (one 512-thread CTA per SM, all of its shared memory), then small ends
+    // (ctas_S CTAs of 256 threads per SM)
+    if (n_M > 0) {
+        const int grid = std::min<int64_t>((int64_t)ctx->n_sm, n_M);
+        k_smem<512><<<grid, 512, ctx->bytes_M, st>>>(
+            list_M, n_M, d_ctr + 5, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
+            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, ctx->bytes_M,
+            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
+            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 7, (GlobalStats *)d_gst);
         CKL();
-        CK(cudaMemcpyAsync(h, d_ctr + 3, 4, cudaMemcpyDeviceToHost, st));
+    }
+    CK(cudaEventRecord(ctx->ev[5], st));
+    if (n_S > 0) {
+        const int grid = std::min<int64_t>((int64_t)ctx->n_sm * ctx->ctas_S, n_S);
+        k_smem<256><<<grid, 256, ctx->bytes_S, st>>>(
+            list_S, n_S, d_ctr + 6, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
+            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, ctx->bytes_S,
+            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
+            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 7, (GlobalStats *)d_gst);
+        CKL();
+    }
+    int n_ovf = 0;
+    if (n_S + n_M > 0) {
+        CK(cudaMemcpyAsync(h, d_ctr + 7, 4, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
         n_ovf = h[0];
-        if (n_ovf) {   // append the overflowed ends to the global list
+        if (n_ovf)   // append the overflowed ends to the global list
             CK(cudaMemcpyAsync(P<int32_t>(ctx->glob_list) + n_glob, ovf_list, (size_t)n_ovf * 4,
                                cudaMemcpyDeviceToDevice, st));
-        }
     }
     CK(cudaEventRecord(ctx->ev[2], st));
     la_status s = run_global(ctx, P<int32_t>(ctx->glob_list), n_glob + n_ovf, nullptr);
@@ -616,9 +648,12 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
     ctx->stats.ms_emit = ms;
     // class counts (host-side tally from the plan counters)
-    ctx->stats.ends_by_class[2] = n_smem - n_ovf;
+    ctx->stats.ends_by_class[2] = n_S + n_M - n_ovf;
     ctx->stats.ends_by_class[3] = n_glob;
     ctx->stats.ends_by_class[4] = n_ovf;
+    ctx->stats.ends_medium = n_M;
+    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[5]);
+    ctx->stats.ms_smem_medium = ms;
     return LA_OK;
 }
 

@@ -66,7 +66,7 @@ def test_c1_single_k(LA, orc):
 
 def test_c2_small_full_schedule(LA, orc):
     r, st = check(LA, orc, cached_batch("C2", scale=0.03), P0)
-    assert st["ends_by_class"][2] > 0
+    assert st["ends_by_class"][2] > 0 and st["ends_medium"] > 0
 
 
 def test_c2_small_forced_global(LA, orc):
@@ -76,7 +76,7 @@ def test_c2_small_forced_global(LA, orc):
 
 def test_c2_small_forced_overflow(LA, orc):
     """Route everything to shared memory: ends whose tables overflow are redone in global memory."""
-    _, st = check(LA, orc, cached_batch("C2", scale=0.03), P0, env={"LA_PRED_DISTINCT": "0.01"})
+    _, st = check(LA, orc, cached_batch("C2", scale=0.03), P0, env={"LA_FORCE_SMEM": "1"})
     assert st["ends_by_class"][4] > 0
 
 
