@@ -371,11 +371,13 @@ def main():
         "contig_ends_per_s": ends_per_s,
         "ends_with_reads_per_s": (ends - st["ends_by_class"][0]) * world * args.steps / (ms_max / 1e3),
         "step_ms": step_ms,
-        "phase_ms": {"smem_kernel": ms_smem, "global_rounds": statistics.mean(s["ms_global"] for s in stats),
+        "phase_ms": {"smem_kernel": ms_smem, "smem_large_tables": statistics.mean(s["ms_smem_medium"] for s in stats),
+                     "global_rounds": statistics.mean(s["ms_global"] for s in stats),
                      "emit": statistics.mean(s["ms_emit"] for s in stats)},
         "work": {"inserts": st["inserts"], "walk_steps": st["walk_steps"], "attempts": st["attempts"],
                  "ext_bases": st["ext_bases"], "ends_by_class": st["ends_by_class"],
-                 "global_rounds": st["global_rounds"]},
+                 "global_rounds": st["global_rounds"], "ends_medium": st["ends_medium"],
+                 "inserts_smem": st["inserts_smem"]},
         "roofline": roof,
         "roofline_hbm": {"bound": "hbm", "achieved": hbm_bytes / (ms_max / args.steps / 1e3) / 1e9,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s",

@@ -78,12 +78,18 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
     return x;
 }
 
-// Hash of a k-mer; the hash function does not affect results (reading #17).
+// Hash of a k-mer: polynomial combine of the words + murmur3 fmix64.  The hash function does not
+// affect results (reading #17), only probe lengths and filter false positives.
 __device__ __forceinline__ uint64_t hash_kmer(const Kmer &K, int KW) {
-    uint64_t h = 0x9E3779B97F4A7C15ull;
+    uint64_t h = K.w[0];
 #pragma unroll
-    for (int w = 0; w < MAX_KW; ++w)
-        if (w < KW) h = mix64(h ^ K.w[w]);
+    for (int w = 1; w < MAX_KW; ++w)
+        if (w < KW) h = h * 0x9E3779B97F4A7C15ull + K.w[w];
+    h ^= h >> 33;
+    h *= 0xff51afd7ed558ccdull;
+    h ^= h >> 33;
+    h *= 0xc4ceb9fe1a85ec53ull;
+    h ^= h >> 33;
     return h;
 }
 

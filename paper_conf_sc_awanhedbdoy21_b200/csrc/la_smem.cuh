@@ -24,11 +24,11 @@
 
 namespace la {
 
-enum : int { CLS_NOREADS = 0, CLS_SHORT = 1, CLS_S = 2, CLS_M = 3, CLS_GLOBAL = 4 };
+enum : int { CLS_NOREADS = 0, CLS_SHORT = 1, CLS_S = 2, CLS_GLOBAL = 7 };   // CLS_S + class index
 constexpr float SMEM_MAX_LOAD = 0.70f;
 
 // ---- shared-memory layout ------------------------------------------------------------------------
-struct SmemFixed {            // per end: staged reads, lengths, walk buffers
+struct SmemFixed {            // per end: staged reads, lengths (+ has-N bit 15), walk buffers
     uint32_t off_qc, off_len, off_walk, off_var, var_bytes;
 };
 
@@ -43,16 +43,21 @@ __host__ __device__ __forceinline__ SmemFixed smem_fixed(int r, int SW, int W, u
     return F;
 }
 
-struct SmemTab {              // per attempt: [vis bits][B1][B2][keys u64][cnts u64]
+// Two slot formats.  INLINE (k <= 63): the 2-bit k-mer itself, 16 B, claimed with one 128-bit CAS;
+// REF (k >= 64): 8 B tag|read|pos, verified against the staged read.  Both + 8 B counters.
+__host__ __device__ __forceinline__ bool inline_keys(int k) { return k <= 63; }
+__host__ __device__ __forceinline__ uint32_t key_bytes(int k) { return inline_keys(k) ? 16u : 8u; }
+
+struct SmemTab {              // per attempt: [vis bits][B1][B2][keys][cnts u64]
     uint32_t off_vis, off_b1, off_b2, off_keys, off_cnts, cap, mwords;
 };
 
 // U = voting-occurrence upper bound (sum over reads of max(0, len-k)).
 __host__ __device__ __forceinline__ SmemTab smem_tab(uint32_t off_var, uint32_t var_bytes, uint32_t U,
-                                                     bool allow_filter) {
+                                                     bool allow_filter, uint32_t kbytes) {
     SmemTab T;
-    // unfiltered: 16 B per slot + 1 visited bit
-    uint32_t cap_nf = (uint32_t)(((uint64_t)var_bytes * 8u) / 129u) & ~1u;
+    const uint32_t per_slot_bits = 8u * (kbytes + 8u) + 1u;   // key + counters + 1 visited bit
+    uint32_t cap_nf = (uint32_t)(((uint64_t)var_bytes * 8u) / per_slot_bits) & ~1u;
     uint32_t mwords = 0;
     uint32_t cap = cap_nf;
     if (allow_filter && (float)U > SMEM_MAX_LOAD * (float)cap_nf) {
@@ -62,7 +67,7 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(uint32_t off_var, uint32_t 
         if (mwords > maxw) mwords = maxw;
         mwords = (mwords + 3u) & ~3u;
         const uint32_t rem = var_bytes > 8u * mwords ? var_bytes - 8u * mwords : 0u;
-        cap = (uint32_t)(((uint64_t)rem * 8u) / 129u) & ~1u;
+        cap = (uint32_t)(((uint64_t)rem * 8u) / per_slot_bits) & ~1u;
     }
     T.cap = cap;
     T.mwords = mwords;
@@ -70,7 +75,7 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(uint32_t off_var, uint32_t 
     T.off_b1 = (off_var + ((cap + 31u) / 32u) * 4u + 15u) & ~15u;
     T.off_b2 = T.off_b1 + mwords * 4u;
     T.off_keys = (T.off_b2 + mwords * 4u + 15u) & ~15u;
-    T.off_cnts = T.off_keys + cap * 8u;
+    T.off_cnts = T.off_keys + cap * kbytes;
     return T;
 }
 
@@ -82,25 +87,32 @@ __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
     return r < 50 ? 0.30f : (r < 200 ? 0.16f : 0.10f);
 }
 
-__device__ __forceinline__ bool fits(int64_t r, int64_t U, int SW, const DevParams &P, uint32_t bytes) {
+__device__ __forceinline__ bool fits(int64_t r, int64_t U, int SW, const DevParams &P, uint32_t bytes,
+                                     uint32_t min_cap) {
     if (bytes == 0) return false;
     const SmemFixed F = smem_fixed((int)r, SW, P.W, bytes);
     if (F.var_bytes == 0) return false;
-    const SmemTab T = smem_tab(F.off_var, F.var_bytes, (uint32_t)U, P.V >= 2);
-    if (T.cap < 512) return false;
+    const SmemTab T = smem_tab(F.off_var, F.var_bytes, (uint32_t)U, P.V >= 2, key_bytes(P.k_min));
+    if (T.cap < min_cap) return false;
     if (T.mwords == 0) return true;   // U <= 0.7 cap: cannot overflow
     return filtered_fraction(r) * (float)U + 64.f <= SMEM_MAX_LOAD * (float)T.cap;
 }
 
+// Shared-memory classes, smallest CTA first: (threads, CTAs/SM) = (64, 12), (128, 6), (256, 3),
+// (256, 2), (512, 1).  Smaller ends get smaller CTAs, so the single-thread walk idles fewer warps;
+// the first class whose table is predicted to fit wins; G = global-memory rounds.
+constexpr int N_SMEM_CLASSES = 5;
+struct PlanBytes {
+    uint32_t b[N_SMEM_CLASSES];   // dynamic shared memory per CTA
+    uint32_t t[N_SMEM_CLASSES];   // threads per CTA
+};
+
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
-                       const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW,
-                       uint32_t bytes_S, uint32_t bytes_M, int32_t *__restrict__ cls,
-                       int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
-                       uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
-                       int32_t *__restrict__ list_S, uint32_t *__restrict__ key_S,
-                       int32_t *__restrict__ list_M, uint32_t *__restrict__ key_M,
-                       int32_t *__restrict__ list_G, int *__restrict__ ctr) {
-    // ctr: [0] n_S [1] n_M [2] n_G [3] NOREADS [4] SHORT
+                       const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW, PlanBytes pb,
+                       int32_t *__restrict__ cls, int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
+                       uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att, int32_t *__restrict__ lists,
+                       uint32_t *__restrict__ keys, int32_t *__restrict__ list_G, int *__restrict__ ctr) {
+    // ctr: [0..4] n per smem class, [5] n_G, [6] NOREADS, [7] SHORT
     const int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (e >= n_ends) return;
     const int64_t r = eoff[e + 1] - eoff[e];
@@ -112,20 +124,24 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         int64_t U = sumlen - r * (int64_t)P.k_min;   // occurrences at the smallest k of the schedule
         if (U < 0) U = 0;
         c = CLS_GLOBAL;
-        if (r < 65536 && U < (1ll << 31)) {
-            if (fits(r, U, SW, P, bytes_S)) c = CLS_S;
-            else if (fits(r, U, SW, P, bytes_M)) c = CLS_M;
-        }
+        int sc = -1;
+        if (r < 65536 && U < (1ll << 30))
+            for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
+                if (fits(r, U, SW, P, pb.b[i], 4u * pb.t[i])) sc = i;
         int64_t U0 = sumlen - r * (int64_t)P.k_start;   // LPT key: occurrences at k_start
         U0 = U0 < 0 ? 0 : (U0 > 0xffffffffll ? 0xffffffffll : U0);
-        const uint32_t key = (uint32_t)U0;
-        if (c == CLS_S) { int i = atomicAdd(&ctr[0], 1); list_S[i] = (int32_t)e; key_S[i] = key; }
-        else if (c == CLS_M) { int i = atomicAdd(&ctr[1], 1); list_M[i] = (int32_t)e; key_M[i] = key; }
-        else { int i = atomicAdd(&ctr[2], 1); list_G[i] = (int32_t)e; }
+        if (sc >= 0) {
+            c = CLS_S + sc;
+            const int i = atomicAdd(&ctr[sc], 1);
+            lists[sc * n_ends + i] = (int32_t)e;
+            keys[sc * n_ends + i] = (uint32_t)U0;
+        } else {
+            list_G[atomicAdd(&ctr[N_SMEM_CLASSES], 1)] = (int32_t)e;
+        }
     }
     cls[e] = c;
     if (c == CLS_NOREADS || c == CLS_SHORT) {
-        atomicAdd(&ctr[c == CLS_NOREADS ? 3 : 4], 1);
+        atomicAdd(&ctr[N_SMEM_CLASSES + (c == CLS_NOREADS ? 1 : 2)], 1);
         out_len[e] = 0;
         out_term[e] = c == CLS_NOREADS ? T_NOREADS : T_SHORT;
         out_k[e] = 0;
@@ -134,11 +150,13 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
 }
 
 // ---- table operations ------------------------------------------------------------------------------
+constexpr uint32_t NEXT_NONE = 0x0FFFFFFFu;   // info word: next slot (28 bits) << 4 | visited << 3 | code
+
 struct SmemCtl {
     int end_idx, overflow, nclaim;
     int k, shift, kmax_eff, done, attempts;
     int best_len, best_term, best_k, best_buf;
-    int maxlen, hasN_any;
+    int maxlen;
     unsigned long long U;
     unsigned long long end_ins, end_steps;
     uint32_t start_slot;
@@ -152,61 +170,237 @@ __device__ __forceinline__ uint32_t filt_index(uint64_t h, uint32_t mbits) {
     return (uint32_t)(((h >> 32) * (uint64_t)mbits) >> 32);
 }
 
-__device__ __forceinline__ uint32_t tab_lookup(const uint64_t *keys, uint32_t cap, const Kmer &K, uint64_t h,
-                                               int k, int KW, const uint64_t *sseq, uint32_t rbase, int SW) {
-    const uint64_t tag = tag_of(h);
-    uint32_t s = slot_of(h, cap);
-    for (uint32_t n = 0; n < cap; ++n) {
-        const uint64_t w = keys[s];
-        if (w == 0) return NONE;
-        if ((w & TAG_MASK) == tag) {
-            const Kmer K2 = extract_kmer(sseq + (size_t)(slot_read(w) - rbase) * SW, slot_pos(w), k, KW);
-            if (kmer_eq(K, K2, KW)) return s;
+// 128-bit compare-and-swap in shared memory (ATOMS.CAS.128, sm_90+).  Returns the old value.
+__device__ __forceinline__ void cas128_shared(void *p, uint64_t c0, uint64_t c1, uint64_t n0, uint64_t n1,
+                                              uint64_t &o0, uint64_t &o1) {
+    const unsigned addr = (unsigned)__cvta_generic_to_shared(p);
+    asm volatile(
+        "{\n .reg .b128 d, b, c;\n mov.b128 b, {%2, %3};\n mov.b128 c, {%4, %5};\n"
+        " atom.shared.cas.b128 d, [%6], b, c;\n mov.b128 {%0, %1}, d;\n}"
+        : "=l"(o0), "=l"(o1)
+        : "l"(c0), "l"(c1), "l"(n0), "l"(n1), "r"(addr)
+        : "memory");
+}
+
+__device__ __forceinline__ void ld128_volatile(const uint64_t *p, uint64_t &x, uint64_t &y) {
+    asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];"
+                 : "=l"(x), "=l"(y)
+                 : "r"((unsigned)__cvta_generic_to_shared(p))
+                 : "memory");
+}
+
+// Stored form of an inline key: word 1 is complemented, so a real key never reads (0, 0) = empty
+// (k <= 63 leaves at least two zero pad bits in word 1).
+__device__ __forceinline__ void inline_form(const Kmer &K, int KW, uint64_t &a, uint64_t &b) {
+    a = K.w[0];
+    b = ~(KW >= 2 ? K.w[1] : 0ull);
+}
+
+struct TabCtx {   // what a table operation needs
+    uint64_t *keys;
+    uint32_t *c32;   // per slot: word 0 = lo[4] (8 bits each), word 1 = hi[4]
+    uint32_t cap;
+    const uint64_t *sseq;
+    uint32_t rbase;
+    int SW, k, KW;
+};
+
+template <bool INL>
+__device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const Kmer &K, uint64_t h) {
+    uint32_t s = slot_of(h, T.cap);
+    if (INL) {
+        uint64_t a, b;
+        inline_form(K, T.KW, a, b);
+        const ulonglong2 *kk = (const ulonglong2 *)T.keys;
+        for (uint32_t n = 0; n < T.cap; ++n) {
+            const ulonglong2 w = kk[s];
+            if (w.y == 0) return NONE;
+            if (w.x == a && w.y == b) return s;
+            s = (s + 1 == T.cap) ? 0 : s + 1;
         }
-        s = (s + 1 == cap) ? 0 : s + 1;
+    } else {
+        const uint64_t tag = tag_of(h);
+        for (uint32_t n = 0; n < T.cap; ++n) {
+            const uint64_t w = T.keys[s];
+            if (w == 0) return NONE;
+            if ((w & TAG_MASK) == tag) {
+                const Kmer K2 = extract_kmer(T.sseq + (size_t)(slot_read(w) - T.rbase) * T.SW, slot_pos(w), T.k, T.KW);
+                if (kmer_eq(K, K2, T.KW)) return s;
+            }
+            s = (s + 1 == T.cap) ? 0 : s + 1;
+        }
     }
     return NONE;
 }
 
 // Alg 1 line 5 (kmer_ht.insert) with the vote of the following base.
-__device__ __forceinline__ void tab_insert(uint64_t *keys, unsigned long long *cnts, uint32_t cap,
-                                           const Kmer &K, uint64_t h, int k, int KW, uint32_t rid, int pos,
-                                           uint32_t b, bool hi, const uint64_t *sseq, uint32_t rbase,
-                                           int SW, int *nclaim, int claim_limit, volatile int *ovf) {
-    const uint64_t tag = tag_of(h);
-    uint32_t s = slot_of(h, cap);
-    volatile uint64_t *vk = keys;
-    uint32_t *c32 = (uint32_t *)cnts;   // per slot: word 0 = lo[4] (8 bits each), word 1 = hi[4]
-    for (;;) {
-        uint64_t w = vk[s];
-        bool hit = false;
-        if (w == 0) {
-            if (*ovf) return;
-            const uint64_t mine = make_slot(tag, rid, (uint32_t)pos);
-            const uint64_t old = atomicCAS((unsigned long long *)&keys[s], 0ull, (unsigned long long)mine);
-            if (old == 0) {
-                hit = true;
-                if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
-            } else {
+template <bool INL>
+__device__ __forceinline__ void tab_insert(const TabCtx &T, const Kmer &K, uint64_t h, uint32_t rid, int pos,
+                                           uint32_t b, bool hi, int *nclaim, int claim_limit, volatile int *ovf) {
+    uint32_t s = slot_of(h, T.cap);
+    bool hit = false;
+    if (INL) {
+        uint64_t a, bb;
+        inline_form(K, T.KW, a, bb);
+        for (;;) {
+            uint64_t x, y;
+            ld128_volatile(&T.keys[2 * s], x, y);
+            if (y == 0) {   // looks empty: the CAS either claims it or returns its true content
+                if (*ovf) return;
+                cas128_shared((void *)&T.keys[2 * s], 0ull, 0ull, a, bb, x, y);
+                if (y == 0) {   // claimed
+                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
+                    break;
+                }
+            } else if (y == bb && x != a) {
+                // a 16 B load is not guaranteed single-copy atomic: if it raced with the claiming CAS,
+                // word 0 may be stale — re-read it (the slot never changes once claimed)
+                x = *(volatile uint64_t *)&T.keys[2 * s];
+            }
+            if (x == a && y == bb) break;
+            s = (s + 1 == T.cap) ? 0 : s + 1;
+        }
+    } else {
+        const uint64_t tag = tag_of(h);
+        volatile uint64_t *vk = T.keys;
+        for (;;) {
+            uint64_t w = vk[s];
+            if (w == 0) {
+                if (*ovf) return;
+                const uint64_t mine = make_slot(tag, rid, (uint32_t)pos);
+                const uint64_t old = atomicCAS((unsigned long long *)&T.keys[s], 0ull, (unsigned long long)mine);
+                if (old == 0) {
+                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
+                    break;
+                }
                 w = old;
             }
+            if ((w & TAG_MASK) == tag) {
+                const Kmer K2 = extract_kmer(T.sseq + (size_t)(slot_read(w) - T.rbase) * T.SW, slot_pos(w), T.k, T.KW);
+                if (kmer_eq(K, K2, T.KW)) break;
+            }
+            s = (s + 1 == T.cap) ? 0 : s + 1;
         }
-        if (!hit && (w & TAG_MASK) == tag) {
-            const Kmer K2 = extract_kmer(sseq + (size_t)(slot_read(w) - rbase) * SW, slot_pos(w), k, KW);
-            hit = kmer_eq(K, K2, KW);
+    }
+    (void)hit;
+    // 32-bit ATOMS.ADD (a 64-bit shared-memory add compiles to a CAS loop)
+    const uint32_t old = atomicAdd(&T.c32[2 * s], 1u << (8 * b));
+    if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit lo counter would carry
+    if (hi) atomicAdd(&T.c32[2 * s + 1], 1u << (8 * b));  // hi <= lo: cannot carry first
+}
+
+// Every voting occurrence of the staged reads: thread per (read, 16-position segment), rolling k-mer,
+// the following base / quality class read from a two-word window.  f(K, j, p, nb, nq2) per occurrence.
+template <int BLOCK, typename F>
+__device__ __forceinline__ unsigned long long for_each_vote(const uint64_t *sseq, const uint64_t *sqc,
+                                                            const uint16_t *slen, int r, int SW, int k, int KW,
+                                                            int maxlen, const volatile int *stop, F &&f) {
+    unsigned long long n = 0;
+    if (maxlen <= k) return 0;
+    const int nseg = (maxlen - k + 15) >> 4;
+    const int items = r * nseg;
+    for (int it = threadIdx.x; it < items; it += BLOCK) {
+        if (*stop) break;
+        const int j = it / nseg;
+        const int sg = it - j * nseg;
+        const uint32_t lf = slen[j];
+        const int len = (int)(lf & 0x7fffu);
+        const int p0 = sg << 4;
+        const int p1 = min(p0 + 16, len - k);
+        if (p0 >= p1) continue;
+        n += (unsigned)(p1 - p0);
+        const uint64_t *R = sseq + (size_t)j * SW;
+        const uint64_t *Q = sqc + (size_t)j * SW;
+        Kmer K = extract_kmer(R, p0, k, KW);
+        int lastN = -1;
+        if (lf & 0x8000u)   // this read has an N
+            for (int i = p0; i < p0 + k; ++i)
+                if (get2(Q, i) == 3u) lastN = i;
+        const int q0 = (p0 + k) >> 5;
+        const uint64_t Ra = R[q0], Rb = R[q0 + 1], Qa = Q[q0], Qb = Q[q0 + 1];
+        for (int p = p0; p < p1; ++p) {
+            const int i = p + k;
+            const bool second = (i >> 5) != q0;
+            const int sh = 62 - ((i & 31) << 1);
+            const uint32_t nb = (uint32_t)((second ? Rb : Ra) >> sh) & 3u;
+            const uint32_t nq = (uint32_t)((second ? Qb : Qa) >> sh) & 3u;
+            if (nq - 1u < 2u && lastN < p) f(K, j, p, nb, nq == 2u);
+            if (nq == 3u) lastN = i;
+            roll_kmer(K, k, KW, nb);
         }
-        if (hit) {   // 32-bit ATOMS.ADD (a 64-bit smem add would be a CAS loop)
-            const uint32_t old = atomicAdd(&c32[2 * s], 1u << (8 * b));
-            if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // 8-bit lo counter would carry
-            if (hi) atomicAdd(&c32[2 * s + 1], 1u << (8 * b));    // hi <= lo: cannot carry first
-            return;
+    }
+    return n;
+}
+
+// Build (filter pass when planned, then insert) and link one attempt.  Returns via C.overflow.
+template <int BLOCK, bool INL>
+__device__ __forceinline__ void build_and_link(SmemCtl &C, const TabCtx &T, uint32_t *B1, uint32_t *B2,
+                                               uint32_t mbits, const uint16_t *slen, const uint64_t *sqc, int r,
+                                               int maxlen, uint32_t r0, const DevParams &P,
+                                               unsigned long long &my_ins) {
+    const volatile int *stop = &C.overflow;
+    const int k = T.k, KW = T.KW;
+    // ---- filter pass: B1 = seen once, B2 = seen at least twice (readings #4) ----
+    if (mbits) {
+        for_each_vote<BLOCK>(T.sseq, sqc, slen, r, T.SW, k, KW, maxlen, stop,
+                             [&](const Kmer &K, int, int, uint32_t, bool) {
+                                 const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
+                                 const uint32_t bit = 1u << (fi & 31);
+                                 if (!(B2[fi >> 5] & bit)) {
+                                     const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                     if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                                 }
+                             });
+        __syncthreads();
+    }
+    // ---- build (Alg 1) ----
+    const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
+    my_ins = for_each_vote<BLOCK>(T.sseq, sqc, slen, r, T.SW, k, KW, maxlen, stop,
+                                  [&](const Kmer &K, int j, int p, uint32_t nb, bool hi) {
+                                      const uint64_t h = hash_kmer(K, KW);
+                                      if (mbits) {
+                                          const uint32_t fi = filt_index(h, mbits);
+                                          if (!((B2[fi >> 5] >> (fi & 31)) & 1u)) return;
+                                      }
+                                      tab_insert<INL>(T, K, h, r0 + (uint32_t)j, p, nb, hi, &C.nclaim,
+                                                      claim_limit, &C.overflow);
+                                  });
+    __syncthreads();
+    if (C.overflow) return;
+    // ---- ext rule + successor links (a5) ----
+    for (uint32_t s = threadIdx.x; s < T.cap; s += BLOCK) {
+        Kmer K;
+        if (INL) {
+            const ulonglong2 w = ((const ulonglong2 *)T.keys)[s];
+            if (w.y == 0) continue;
+            K.w[0] = w.x;
+            K.w[1] = KW >= 2 ? ~w.y : 0ull;
+            K.w[2] = K.w[3] = 0;
+        } else {
+            const uint64_t w = T.keys[s];
+            if (w == 0) continue;
+            K = extract_kmer(T.sseq + (size_t)(slot_read(w) - T.rbase) * T.SW, slot_pos(w), k, KW);
         }
-        s = (s + 1 == cap) ? 0 : s + 1;
+        const uint32_t lw = T.c32[2 * s], hw = T.c32[2 * s + 1];
+        uint32_t lo[4], hi[4];
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+            lo[b] = (lw >> (8 * b)) & 0xffu;
+            hi[b] = (hw >> (8 * b)) & 0xffu;
+        }
+        const int code = ext_rule(lo, hi, P.V, P.F);
+        uint32_t nxt = NEXT_NONE;
+        if (code < 4) {
+            roll_kmer(K, k, KW, (uint32_t)code);
+            const uint32_t t = tab_lookup<INL>(T, K, hash_kmer(K, KW));
+            nxt = t == NONE ? NEXT_NONE : t;
+        }
+        T.c32[2 * s] = (nxt << 4) | (uint32_t)code;
     }
 }
 
 template <int BLOCK>
-__global__ void __launch_bounds__(BLOCK, BLOCK >= 512 ? 1 : 3) k_smem(
+__global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_smem(
     const int32_t *__restrict__ list, int n_list, int *__restrict__ work_ctr,
     const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
     const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
@@ -232,42 +426,33 @@ __global__ void __launch_bounds__(BLOCK, BLOCK >= 512 ? 1 : 3) k_smem(
         const int64_t r0 = eoff[e];
         const int r = (int)(eoff[e + 1] - r0);
         const SmemFixed FX = smem_fixed(r, SW, P.W, smem_bytes);
+        if (FX.var_bytes < 4096u) {   // reads do not fit: the global path takes this end
+            if (tid == 0) ovf_list[atomicAdd(n_ovf, 1)] = e;
+            continue;
+        }
         uint64_t *sseq = (uint64_t *)sm;
         uint64_t *sqc = (uint64_t *)(sm + FX.off_qc);
         uint16_t *slen = (uint16_t *)(sm + FX.off_len);
         uint8_t *swalk = sm + FX.off_walk;   // two buffers of Wp bytes
         const int Wp = (P.W + 15) & ~15;
-        if (FX.var_bytes < 2048u) {   // reads do not fit at all: the global path takes this end
-            if (tid == 0) ovf_list[atomicAdd(n_ovf, 1)] = e;
-            continue;
-        }
 
         // stage the end's packed reads (contiguous in HBM): coalesced 16 B loads
         {
             const int nw = r * SW;
-            if ((SW & 1) == 0) {
-                const uint4 *gs = (const uint4 *)(rseq + r0 * SW);
-                const uint4 *gq = (const uint4 *)(rqc + r0 * SW);
-                uint4 *ss = (uint4 *)sseq;
-                uint4 *sq = (uint4 *)sqc;
-                for (int i = tid; i < nw / 2; i += BLOCK) { ss[i] = gs[i]; sq[i] = gq[i]; }
-            } else {
-                for (int i = tid; i < nw; i += BLOCK) { sseq[i] = rseq[r0 * SW + i]; sqc[i] = rqc[r0 * SW + i]; }
-            }
-            int ml = 0, hn = 0;
+            const uint4 *gs = (const uint4 *)(rseq + r0 * SW);
+            const uint4 *gq = (const uint4 *)(rqc + r0 * SW);
+            uint4 *ss = (uint4 *)sseq;
+            uint4 *sq = (uint4 *)sqc;
+            for (int i = tid; i < nw / 2; i += BLOCK) { ss[i] = gs[i]; sq[i] = gq[i]; }   // SW is even
+            int ml = 0;
             for (int i = tid; i < r; i += BLOCK) {
                 const int l = rlen[r0 + i];
-                slen[i] = (uint16_t)l;
+                slen[i] = (uint16_t)(l | (rflag[r0 + i] ? 0x8000 : 0));
                 ml = max(ml, l);
-                hn |= rflag[r0 + i];
             }
-            for (int o = 16; o; o >>= 1) {
-                ml = max(ml, __shfl_xor_sync(0xffffffffu, ml, o));
-                hn |= __shfl_xor_sync(0xffffffffu, hn, o);
-            }
+            for (int o = 16; o; o >>= 1) ml = max(ml, __shfl_xor_sync(0xffffffffu, ml, o));
             if (tid == 0) {
                 C.maxlen = 0;
-                C.hasN_any = 0;
                 C.kmax_eff = min(P.k_max, (int)clen[e]);
                 C.k = P.k_start;
                 C.shift = 0;
@@ -282,152 +467,63 @@ __global__ void __launch_bounds__(BLOCK, BLOCK >= 512 ? 1 : 3) k_smem(
                 C.end_steps = 0;
             }
             __syncthreads();
-            if (lane == 0) { atomicMax(&C.maxlen, ml); atomicOr(&C.hasN_any, hn); }
+            if (lane == 0) atomicMax(&C.maxlen, ml);
         }
         __syncthreads();
         const int maxlen = C.maxlen;
-        const bool anyN = C.hasN_any != 0;
 
         // ---------------- retry loop ----------------
         for (;;) {
             const int k = C.k;
             const int KW = kwords(k);
+            const bool INL = inline_keys(k);
             // voting-occurrence bound at this k -> table plan
             {
                 unsigned long long u = 0;
-                for (int i = tid; i < r; i += BLOCK) u += (unsigned)max(0, (int)slen[i] - k);
+                for (int i = tid; i < r; i += BLOCK) u += (unsigned)max(0, (int)(slen[i] & 0x7fff) - k);
                 for (int o = 16; o; o >>= 1) u += __shfl_xor_sync(0xffffffffu, u, o);
                 if (tid == 0) C.U = 0;
                 __syncthreads();
                 if (lane == 0 && u) atomicAdd(&C.U, u);
                 __syncthreads();
             }
-            const uint32_t U = (uint32_t)C.U;
-            const SmemTab T = smem_tab(FX.off_var, FX.var_bytes, U, P.V >= 2);
-            const uint32_t cap = T.cap;
-            if (cap < 128u) {   // no room for a table at this k
+            const SmemTab TB = smem_tab(FX.off_var, FX.var_bytes, (uint32_t)C.U, P.V >= 2, key_bytes(k));
+            const uint32_t cap = TB.cap;
+            if (cap < 4u * BLOCK) {   // no room for a table at this k (keeps claims + in-flight < cap)
                 if (tid == 0) C.overflow = 1;
                 __syncthreads();
                 break;
             }
-            const uint32_t mbits = T.mwords * 32u;
-            uint32_t *svis = (uint32_t *)(sm + T.off_vis);
-            uint32_t *B1 = (uint32_t *)(sm + T.off_b1);
-            uint32_t *B2 = (uint32_t *)(sm + T.off_b2);
-            uint64_t *keys = (uint64_t *)(sm + T.off_keys);
-            unsigned long long *cnts = (unsigned long long *)(sm + T.off_cnts);
-            // clear keys, counters, visited bits and filters
+            const uint32_t mbits = TB.mwords * 32u;
+            uint32_t *svis = (uint32_t *)(sm + TB.off_vis);
+            (void)svis;
+            uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);
+            uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
+            TabCtx T;
+            T.keys = (uint64_t *)(sm + TB.off_keys);
+            T.c32 = (uint32_t *)(sm + TB.off_cnts);
+            T.cap = cap;
+            T.sseq = sseq;
+            T.rbase = (uint32_t)r0;
+            T.SW = SW;
+            T.k = k;
+            T.KW = KW;
+            // clear keys + counters (contiguous) and the filters
             {
                 const uint4 z = make_uint4(0, 0, 0, 0);
-                uint4 *a = (uint4 *)keys;
-                for (uint32_t i = tid; i < cap; i += BLOCK) a[i] = z;   // keys + cnts: 16 B per slot
-                for (uint32_t i = tid; i < (cap + 31u) / 32u; i += BLOCK) svis[i] = 0;
-                for (uint32_t i = tid; i < 2u * T.mwords; i += BLOCK) B1[i] = 0;   // B1, B2 contiguous
+                uint4 *a = (uint4 *)T.keys;
+                const uint32_t n16 = (cap * (key_bytes(k) + 8u)) / 16u;
+                for (uint32_t i = tid; i < n16; i += BLOCK) a[i] = z;
+                for (uint32_t i = tid; i < 2u * TB.mwords; i += BLOCK) B1[i] = 0;   // B1, B2 contiguous
                 if (tid == 0) C.nclaim = 0;
             }
             __syncthreads();
-
-            const int nseg = maxlen > k ? ((maxlen - k + 15) >> 4) : 0;
-            const int items = r * nseg;
-
-            // ---- filter pass: B1 = seen once, B2 = seen at least twice ----
-            if (mbits) {
-                for (int it = tid; it < items; it += BLOCK) {
-                    const int j = it / nseg;
-                    const int sg = it - j * nseg;
-                    const int len = slen[j];
-                    const int p0 = sg << 4;
-                    const int p1 = min(p0 + 16, len - k);
-                    if (p0 >= p1) continue;
-                    const uint64_t *R = sseq + (size_t)j * SW;
-                    const uint64_t *Q = sqc + (size_t)j * SW;
-                    Kmer K = extract_kmer(R, p0, k, KW);
-                    int lastN = -1;
-                    if (anyN)
-                        for (int i = p0; i < p0 + k; ++i)
-                            if (get2(Q, i) == 3u) lastN = i;
-                    for (int p = p0; p < p1; ++p) {
-                        const uint32_t nb = get2(R, p + k);
-                        const uint32_t nq = get2(Q, p + k);
-                        if ((nq == 1u || nq == 2u) && lastN < p) {
-                            const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
-                            const uint32_t bit = 1u << (fi & 31);
-                            if (!(B2[fi >> 5] & bit)) {
-                                const uint32_t old = atomicOr(&B1[fi >> 5], bit);
-                                if (old & bit) atomicOr(&B2[fi >> 5], bit);
-                            }
-                        }
-                        if (nq == 3u) lastN = p + k;
-                        roll_kmer(K, k, KW, nb);
-                    }
-                }
-                __syncthreads();
-            }
-
-            // ---- build (Alg 1) ----
             unsigned long long my_ins = 0;
-            {
-                const int claim_limit = (int)(SMEM_MAX_LOAD * (float)cap);
-                for (int it = tid; it < items; it += BLOCK) {
-                    if (*(volatile int *)&C.overflow) break;
-                    const int j = it / nseg;
-                    const int sg = it - j * nseg;
-                    const int len = slen[j];
-                    const int p0 = sg << 4;
-                    const int p1 = min(p0 + 16, len - k);
-                    if (p0 >= p1) continue;
-                    my_ins += (unsigned)(p1 - p0);
-                    const uint64_t *R = sseq + (size_t)j * SW;
-                    const uint64_t *Q = sqc + (size_t)j * SW;
-                    Kmer K = extract_kmer(R, p0, k, KW);
-                    int lastN = -1;
-                    if (anyN)
-                        for (int i = p0; i < p0 + k; ++i)
-                            if (get2(Q, i) == 3u) lastN = i;
-                    for (int p = p0; p < p1; ++p) {
-                        const uint32_t nb = get2(R, p + k);
-                        const uint32_t nq = get2(Q, p + k);
-                        if ((nq == 1u || nq == 2u) && lastN < p) {
-                            const uint64_t h = hash_kmer(K, KW);
-                            bool keep = true;
-                            if (mbits) {
-                                const uint32_t fi = filt_index(h, mbits);
-                                keep = (B2[fi >> 5] >> (fi & 31)) & 1u;
-                            }
-                            if (keep)
-                                tab_insert(keys, cnts, cap, K, h, k, KW, (uint32_t)(r0 + j), p, nb, nq == 2u, sseq,
-                                           (uint32_t)r0, SW, &C.nclaim, claim_limit, &C.overflow);
-                        }
-                        if (nq == 3u) lastN = p + k;
-                        roll_kmer(K, k, KW, nb);
-                    }
-                }
-            }
+            if (INL) build_and_link<BLOCK, true>(C, T, B1, B2, mbits, slen, sqc, r, maxlen, (uint32_t)r0, P, my_ins);
+            else build_and_link<BLOCK, false>(C, T, B1, B2, mbits, slen, sqc, r, maxlen, (uint32_t)r0, P, my_ins);
+            if (C.overflow) break;   // uniform: read after build_and_link's barrier
             for (int o = 16; o; o >>= 1) my_ins += __shfl_xor_sync(0xffffffffu, my_ins, o);
             if (lane == 0 && my_ins) atomicAdd(&C.end_ins, my_ins);
-            __syncthreads();
-            if (C.overflow) break;
-
-            // ---- ext rule + successor links (a5): info = next_slot << 3 | code ----
-            for (uint32_t s = tid; s < cap; s += BLOCK) {
-                const uint64_t w = keys[s];
-                if (w == 0) continue;
-                const unsigned long long c8 = cnts[s];
-                uint32_t lo[4], hi[4];
-#pragma unroll
-                for (int b = 0; b < 4; ++b) {
-                    lo[b] = (uint32_t)(c8 >> (8 * b)) & 0xffu;
-                    hi[b] = (uint32_t)(c8 >> (32 + 8 * b)) & 0xffu;
-                }
-                const int code = ext_rule(lo, hi, P.V, P.F);
-                uint32_t nxt = NONE;
-                if (code < 4) {
-                    Kmer K = extract_kmer(sseq + (size_t)(slot_read(w) - (uint32_t)r0) * SW, slot_pos(w), k, KW);
-                    roll_kmer(K, k, KW, (uint32_t)code);
-                    nxt = tab_lookup(keys, cap, K, hash_kmer(K, KW), k, KW, sseq, (uint32_t)r0, SW);
-                }
-                cnts[s] = (unsigned long long)((nxt << 3) | (uint32_t)code);
-            }
             if (tid == 0) {
                 // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
                 const uint64_t *Tl = tail + (size_t)e * TAIL_W;
@@ -442,33 +538,30 @@ __global__ void __launch_bounds__(BLOCK, BLOCK >= 512 ? 1 : 3) k_smem(
 #pragma unroll
                     for (int i = 0; i < TAIL_W; ++i) Tw[i] = Tl[i];
                     const Kmer K = extract_kmer(Tw, p, k, KW);
-                    C.start_slot = tab_lookup(keys, cap, K, hash_kmer(K, KW), k, KW, sseq, (uint32_t)r0, SW);
+                    const uint64_t h = hash_kmer(K, KW);
+                    C.start_slot = INL ? tab_lookup<true>(T, K, h) : tab_lookup<false>(T, K, h);
                 }
             }
             __syncthreads();
 
-            // ---- walk (Alg 2) + retry decision, one thread ----
+            // ---- walk (Alg 2) over the successor links + retry decision, one thread ----
             if (tid == 0) {
                 uint8_t *wb = swalk + (C.best_buf ^ 1) * Wp;
-                uint32_t node = C.start_slot;
+                uint32_t *info = T.c32;   // info word of slot s at info[2 s]
+                uint32_t node = C.start_slot == NONE ? NEXT_NONE : C.start_slot;
                 int len = 0, term = T_MAXLEN;
                 unsigned long long steps = 0;
-                const uint32_t *info = (const uint32_t *)cnts;   // low word of each 8 B counter slot
                 for (int i = 0; i < P.W; ++i) {
-                    if (node != NONE) {   // loop check before lookup (Alg 2 lines 6-8)
-                        const uint32_t bit = 1u << (node & 31);
-                        const uint32_t v = svis[node >> 5];
-                        if (v & bit) { term = T_LOOP; break; }
-                        svis[node >> 5] = v | bit;
-                    }
-                    ++steps;
-                    if (node == NONE) { term = T_DEADEND; break; }
+                    ++steps;   // a lookup (the loop check of a present k-mer precedes it, below)
+                    if (node == NEXT_NONE) { term = T_DEADEND; break; }
                     const uint32_t inf = info[2 * node];
+                    if (inf & 8u) { term = T_LOOP; --steps; break; }   // visited: loop check before lookup
+                    info[2 * node] = inf | 8u;
                     const uint32_t code = inf & 7u;
                     if (code == CODE_FORK) { term = T_FORK; break; }
                     if (code == CODE_DEADEND) { term = T_DEADEND; break; }
                     wb[len++] = "ACGT"[code];
-                    node = inf >> 3;
+                    node = inf >> 4;
                 }
                 C.attempts += 1;
                 C.end_steps += steps;

@@ -61,8 +61,9 @@ struct la_ctx {
     bool loaded = false;
     std::string err;
     int n_sm = 148;
-    int ctas_S = 3;               // small-table CTAs per SM
-    uint32_t bytes_S = 0, bytes_M = 0;   // dynamic shared memory per CTA: small / medium kernel
+    int cls_threads[N_SMEM_CLASSES] = {64, 128, 256, 256, 512};
+    int cls_ctas[N_SMEM_CLASSES] = {12, 6, 3, 2, 1};   // resident CTAs per SM of each shared-memory class
+    uint32_t cls_bytes[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};   // dynamic shared memory per CTA
     la_params params{};
     DevParams dp{};
     Encoded enc, spare;   // current encoding; la_load_batch fills `spare` and swaps on success
@@ -173,12 +174,12 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     cudaDeviceProp prop;
     cudaGetDeviceProperties(&prop, device);
     ctx->n_sm = prop.multiProcessorCount;
-    if (const char *s = getenv("LA_SMEM_CTAS")) ctx->ctas_S = std::max(1, atoi(s));
     // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
-    size_t per = prop.sharedMemPerMultiprocessor / ctx->ctas_S - 1024 - 512 /* static */;
-    per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - 512);
-    ctx->bytes_S = (uint32_t)(per & ~(size_t)127);
-    ctx->bytes_M = (uint32_t)((prop.sharedMemPerBlockOptin - 512) & ~(size_t)127);
+    for (int i = 0; i < N_SMEM_CLASSES; ++i) {
+        size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - 512 /* static */;
+        per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - 512);
+        ctx->cls_bytes[i] = (uint32_t)(per & ~(size_t)127);
+    }
     if (cuda_stream) ctx->stream = (cudaStream_t)cuda_stream;
     else {
         if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) {
@@ -188,8 +189,10 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
-    if (cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->bytes_S) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->bytes_M) != cudaSuccess) {
+    if (cudaFuncSetAttribute(k_smem<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[0]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[1]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[3]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess) {
         cudaGetLastError();
         la_destroy(ctx);
         return LA_ERR_CUDA;
@@ -484,8 +487,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     const int W = std::max(dp.W, 1);
     ctx->stats = la_stats{};
     ctx->g_attempts = 0;
-    ctx->stats.smem_bytes_per_cta = ctx->bytes_S;
-    ctx->stats.smem_ctas_per_sm = ctx->ctas_S;
+    ctx->stats.smem_bytes_per_cta = ctx->cls_bytes[0];
+    ctx->stats.smem_ctas_per_sm = ctx->cls_ctas[0];
 
     CK(grow(ctx->cls, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->out_len, std::max<int64_t>(nE, 1) * 4));
@@ -493,8 +496,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->out_k, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->out_att, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->walk_buf, std::max<int64_t>(nE, 1) * W));
-    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 8));
-    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 8));
+    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4 * N_SMEM_CLASSES));
+    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4 * N_SMEM_CLASSES));
     CK(grow(ctx->smem_list2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
@@ -502,41 +505,46 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->gstats, 64));
     CK(grow(ctx->ext_off, (nE + 1) * 8));
     CK(grow_host(ctx->h_small, 256));
-    int *d_ctr = P<int>(ctx->ctrs);   // [0] n_S [1] n_M [2] n_G [3] NOREADS [4] SHORT [5,6] work [7] n_ovf
+    int *d_ctr = P<int>(ctx->ctrs);   // [0..4] n per class [5] n_G [6] NOREADS [7] SHORT [15] n_ovf [16..20] work
     unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
 
     CK(cudaEventRecord(ctx->ev[0], st));
-    CK(cudaMemsetAsync(d_ctr, 0, 64, st));
+    CK(cudaMemsetAsync(d_ctr, 0, 128, st));
     CK(cudaMemsetAsync(d_gst, 0, 64, st));
     int *h = (int *)ctx->h_small.p;
-    int n_S = 0, n_M = 0, n_glob = 0;
-    int32_t *list_S = P<int32_t>(ctx->smem_list), *list_M = P<int32_t>(ctx->smem_list) + nE;
-    uint32_t *key_S = P<uint32_t>(ctx->smem_key), *key_M = P<uint32_t>(ctx->smem_key) + nE;
+    int ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
+    int n_glob = 0;
+    int32_t *lists = P<int32_t>(ctx->smem_list);
+    uint32_t *keys = P<uint32_t>(ctx->smem_key);
     if (nE) {
         // test hook: force every end with reads onto the global path
         const bool force_global = getenv("LA_FORCE_GLOBAL") && atoi(getenv("LA_FORCE_GLOBAL")) != 0;
         // test hook: pretend every end fits the small-table kernel (exercises the overflow redo)
         const bool force_smem = getenv("LA_FORCE_SMEM") && atoi(getenv("LA_FORCE_SMEM")) != 0;
+        PlanBytes pb;
+        for (int i = 0; i < N_SMEM_CLASSES; ++i) {
+            pb.b[i] = force_global ? 0u : ctx->cls_bytes[i];
+            pb.t[i] = (uint32_t)ctx->cls_threads[i];
+        }
+        if (force_smem) pb.b[0] = 0xffffffffu;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
-            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW,
-            force_global ? 0u : (force_smem ? 0xffffffffu : ctx->bytes_S), force_global ? 0u : ctx->bytes_M,
-            P<int32_t>(ctx->cls), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), list_S, key_S, list_M, key_M, P<int32_t>(ctx->glob_list), d_ctr);
+            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb, P<int32_t>(ctx->cls),
+            P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
+            lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
-        CK(cudaMemcpyAsync(h, d_ctr, 20, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h, d_ctr, 4 * (N_SMEM_CLASSES + 3), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
-        n_S = h[0];
-        n_M = h[1];
-        n_glob = h[2];
-        ctx->stats.ends_by_class[0] = h[3];
-        ctx->stats.ends_by_class[1] = h[4];
+        for (int i = 0; i < N_SMEM_CLASSES; ++i) ncls[i] = h[i];
+        n_glob = h[N_SMEM_CLASSES];
+        ctx->stats.ends_by_class[0] = h[N_SMEM_CLASSES + 1];
+        ctx->stats.ends_by_class[1] = h[N_SMEM_CLASSES + 2];
     }
     // LPT order for the persistent kernels: largest expected work first
-    for (int cls = 0; cls < 2; ++cls) {
-        const int n = cls ? n_M : n_S;
+    for (int c = 0; c < N_SMEM_CLASSES; ++c) {
+        const int n = ncls[c];
         if (n < 2) continue;
-        int32_t *lst = cls ? list_M : list_S;
-        uint32_t *key = cls ? key_M : key_S;
+        int32_t *lst = lists + (size_t)c * nE;
+        uint32_t *key = keys + (size_t)c * nE;
         size_t tb = 0;
         cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, key, P<uint32_t>(ctx->smem_key2), lst,
                                                   P<int32_t>(ctx->smem_list2), n, 0, 32, st);
@@ -548,30 +556,37 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     CK(cudaEventRecord(ctx->ev[1], st));
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
-    // medium ends first (one 512-thread CTA per SM, all of its shared memory), then small ends
-    // (ctas_S CTAs of 256 threads per SM)
-    if (n_M > 0) {
-        const int grid = std::min<int64_t>((int64_t)ctx->n_sm, n_M);
-        k_smem<512><<<grid, 512, ctx->bytes_M, st>>>(
-            list_M, n_M, d_ctr + 5, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
-            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, ctx->bytes_M,
-            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 7, (GlobalStats *)d_gst);
-        CKL();
-    }
-    CK(cudaEventRecord(ctx->ev[5], st));
-    if (n_S > 0) {
-        const int grid = std::min<int64_t>((int64_t)ctx->n_sm * ctx->ctas_S, n_S);
-        k_smem<256><<<grid, 256, ctx->bytes_S, st>>>(
-            list_S, n_S, d_ctr + 6, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
-            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, ctx->bytes_S,
-            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 7, (GlobalStats *)d_gst);
-        CKL();
+    // largest tables first (1 CTA/SM, all shared memory) ... smallest last (12 CTAs/SM)
+    for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
+        const int n = ncls[c];
+        if (n > 0) {
+            const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm * ctx->cls_ctas[c], n);
+            const uint32_t bytes = ctx->cls_bytes[c];
+            int32_t *lst = lists + (size_t)c * nE;
+            int *wc = d_ctr + 16 + c;
+#define LA_LAUNCH_SMEM(B)                                                                                   \
+    k_smem<B><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), \
+                                      P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail),             \
+                                      P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                 \
+                                      P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                       \
+                                      P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                         \
+                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst)
+            switch (ctx->cls_threads[c]) {
+                case 64: LA_LAUNCH_SMEM(64); break;
+                case 128: LA_LAUNCH_SMEM(128); break;
+                case 256: LA_LAUNCH_SMEM(256); break;
+                default: LA_LAUNCH_SMEM(512); break;
+            }
+#undef LA_LAUNCH_SMEM
+            CKL();
+        }
+        if (c == 2) CK(cudaEventRecord(ctx->ev[5], st));   // after the 1- and 2-CTA/SM classes
     }
     int n_ovf = 0;
-    if (n_S + n_M > 0) {
-        CK(cudaMemcpyAsync(h, d_ctr + 7, 4, cudaMemcpyDeviceToHost, st));
+    int n_smem = 0;
+    for (int c = 0; c < N_SMEM_CLASSES; ++c) n_smem += ncls[c];
+    if (n_smem > 0) {
+        CK(cudaMemcpyAsync(h, d_ctr + 15, 4, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
         n_ovf = h[0];
         if (n_ovf)   // append the overflowed ends to the global list
@@ -648,10 +663,10 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
     ctx->stats.ms_emit = ms;
     // class counts (host-side tally from the plan counters)
-    ctx->stats.ends_by_class[2] = n_S + n_M - n_ovf;
+    ctx->stats.ends_by_class[2] = n_smem - n_ovf;
     ctx->stats.ends_by_class[3] = n_glob;
     ctx->stats.ends_by_class[4] = n_ovf;
-    ctx->stats.ends_medium = n_M;
+    ctx->stats.ends_medium = ncls[3] + ncls[4];
     cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[5]);
     ctx->stats.ms_smem_medium = ms;
     return LA_OK;
