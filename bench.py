@@ -376,7 +376,7 @@ def main():
                      "emit": statistics.mean(s["ms_emit"] for s in stats)},
         "work": {"inserts": st["inserts"], "walk_steps": st["walk_steps"], "attempts": st["attempts"],
                  "ext_bases": st["ext_bases"], "ends_by_class": st["ends_by_class"],
-                 "global_rounds": st["global_rounds"], "ends_medium": st["ends_medium"],
+                 "global_rounds": st["global_rounds"], "ends_medium": st["ends_medium"], "ends_xl": st["ends_xl"],
                  "inserts_smem": st["inserts_smem"]},
         "roofline": roof,
         "roofline_hbm": {"bound": "hbm", "achieved": hbm_bytes / (ms_max / args.steps / 1e3) / 1e9,

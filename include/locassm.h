@@ -108,7 +108,9 @@ typedef struct {
     int32_t smem_ctas_per_sm;
     int32_t global_rounds;
     int64_t ends_medium;         /* ends routed to the medium (one CTA per SM) kernel             */
-    double ms_smem_medium;       /* its device time (included in ms_smem)                          */
+    double ms_smem_medium;       /* device time of the XL + 1- and 2-CTA/SM classes (in ms_smem)   */
+    int64_t ends_xl;             /* ends whose table lived in the XL class's global scratch        */
+    int64_t xl_scratch_bytes;
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);

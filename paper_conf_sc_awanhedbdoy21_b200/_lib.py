@@ -46,7 +46,8 @@ class la_stats(ctypes.Structure):
                 ("ends_by_class", ctypes.c_int64 * 5), ("kernel_launches", ctypes.c_int64),
                 ("smem_bytes_per_cta", ctypes.c_int64), ("smem_ctas_per_sm", ctypes.c_int32),
                 ("global_rounds", ctypes.c_int32), ("ends_medium", ctypes.c_int64),
-                ("ms_smem_medium", ctypes.c_double)]
+                ("ms_smem_medium", ctypes.c_double), ("ends_xl", ctypes.c_int64),
+                ("xl_scratch_bytes", ctypes.c_int64)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_get_stats",

@@ -73,7 +73,7 @@ struct la_ctx {
         smem_key2, glob_list, ctrs, ext_off, ext_seq, gstats, cub_tmp;
     DevBuf g_state, g_act, g_act2, g_still, g_cap, g_nrd, g_capoff, g_rdoff, g_slots, g_cnt, g_vis,
         g_cur;
-    DevBuf lens64;
+    DevBuf lens64, xl_scratch;
     HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
     int64_t g_attempts = 0;
     cudaEvent_t ev[6] = {};
@@ -189,10 +189,11 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
-    if (cudaFuncSetAttribute(k_smem<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[0]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[1]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[3]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess) {
+    if (cudaFuncSetAttribute(k_smem<64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[0]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[1]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[3]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess ||
+        cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess) {
         cudaGetLastError();
         la_destroy(ctx);
         return LA_ERR_CUDA;
@@ -213,7 +214,7 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
                       &ctx->glob_list, &ctx->ctrs, &ctx->ext_off, &ctx->ext_seq, &ctx->gstats,
                       &ctx->cub_tmp, &ctx->g_state, &ctx->g_act, &ctx->g_act2, &ctx->g_still, &ctx->g_cap,
                       &ctx->g_nrd, &ctx->g_capoff, &ctx->g_rdoff, &ctx->g_slots, &ctx->g_cnt, &ctx->g_vis,
-                      &ctx->g_cur, &ctx->lens64})
+                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch})
         b->release();
     for (HostBuf *b : {&ctx->h_ext_off, &ctx->h_ext_seq, &ctx->h_term, &ctx->h_k, &ctx->h_att, &ctx->h_small})
         b->release();
@@ -496,8 +497,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->out_k, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->out_att, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->walk_buf, std::max<int64_t>(nE, 1) * W));
-    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4 * N_SMEM_CLASSES));
-    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4 * N_SMEM_CLASSES));
+    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4 * (N_SMEM_CLASSES + 1)));
+    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4 * (N_SMEM_CLASSES + 1)));
     CK(grow(ctx->smem_list2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
@@ -513,7 +514,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(cudaMemsetAsync(d_gst, 0, 64, st));
     int *h = (int *)ctx->h_small.p;
     int ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
-    int n_glob = 0;
+    int n_glob = 0, n_xl = 0, xl_umax = 0, xl_rmax = 0;
     int32_t *lists = P<int32_t>(ctx->smem_list);
     uint32_t *keys = P<uint32_t>(ctx->smem_key);
     if (nE) {
@@ -528,20 +529,24 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         }
         if (force_smem) pb.b[0] = 0xffffffffu;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
-            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb, P<int32_t>(ctx->cls),
+            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, pb,
+            (force_global || force_smem) ? 0u : ctx->cls_bytes[N_SMEM_CLASSES - 1], P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
             lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
-        CK(cudaMemcpyAsync(h, d_ctr, 4 * (N_SMEM_CLASSES + 3), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h, d_ctr, 4 * 11, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
         for (int i = 0; i < N_SMEM_CLASSES; ++i) ncls[i] = h[i];
         n_glob = h[N_SMEM_CLASSES];
         ctx->stats.ends_by_class[0] = h[N_SMEM_CLASSES + 1];
         ctx->stats.ends_by_class[1] = h[N_SMEM_CLASSES + 2];
+        n_xl = h[8];
+        xl_umax = h[9];
+        xl_rmax = h[10];
     }
     // LPT order for the persistent kernels: largest expected work first
-    for (int c = 0; c < N_SMEM_CLASSES; ++c) {
-        const int n = ncls[c];
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
+        const int n = c == N_SMEM_CLASSES ? n_xl : ncls[c];
         if (n < 2) continue;
         int32_t *lst = lists + (size_t)c * nE;
         uint32_t *key = keys + (size_t)c * nE;
@@ -556,7 +561,25 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     CK(cudaEventRecord(ctx->ev[1], st));
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
-    // largest tables first (1 CTA/SM, all shared memory) ... smallest last (12 CTAs/SM)
+    // XL (global-scratch tables) first, then the shared-memory classes from the largest tables
+    // (1 CTA/SM, all shared memory) to the smallest (12 CTAs/SM)
+    if (n_xl > 0) {
+        const uint32_t bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
+        const uint32_t icap = smem_fixed(dp.W, bytes, 1u).icap;
+        const uint32_t stride = xl_stride(xl_rmax, xl_umax, dp.V >= 2, icap);
+        const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm, n_xl);
+        CK(grow(ctx->xl_scratch, (size_t)grid * stride));
+        int32_t *lst = lists + (size_t)N_SMEM_CLASSES * nE;
+        k_smem<XL_THREADS, true><<<grid, XL_THREADS, bytes, st>>>(
+            lst, n_xl, d_ctr + 21, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
+            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
+            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
+            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst, P<unsigned char>(ctx->xl_scratch),
+            stride);
+        CKL();
+        ctx->stats.ends_xl = n_xl;
+        ctx->stats.xl_scratch_bytes = (int64_t)grid * stride;
+    }
     for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
         const int n = ncls[c];
         if (n > 0) {
@@ -565,12 +588,12 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
             int32_t *lst = lists + (size_t)c * nE;
             int *wc = d_ctr + 16 + c;
 #define LA_LAUNCH_SMEM(B)                                                                                   \
-    k_smem<B><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), \
+    k_smem<B, false><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), \
                                       P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail),             \
                                       P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                 \
                                       P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                       \
                                       P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                         \
-                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst)
+                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst, nullptr, 0u)
             switch (ctx->cls_threads[c]) {
                 case 64: LA_LAUNCH_SMEM(64); break;
                 case 128: LA_LAUNCH_SMEM(128); break;
@@ -583,7 +606,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         if (c == 2) CK(cudaEventRecord(ctx->ev[5], st));   // after the 1- and 2-CTA/SM classes
     }
     int n_ovf = 0;
-    int n_smem = 0;
+    int n_smem = n_xl;
     for (int c = 0; c < N_SMEM_CLASSES; ++c) n_smem += ncls[c];
     if (n_smem > 0) {
         CK(cudaMemcpyAsync(h, d_ctr + 15, 4, cudaMemcpyDeviceToHost, st));

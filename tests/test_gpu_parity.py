@@ -66,7 +66,7 @@ def test_c1_single_k(LA, orc):
 
 def test_c2_small_full_schedule(LA, orc):
     r, st = check(LA, orc, cached_batch("C2", scale=0.03), P0)
-    assert st["ends_by_class"][2] > 0 and st["ends_medium"] > 0
+    assert st["ends_by_class"][2] > 0 and st["ends_medium"] > 0 and st["ends_xl"] > 0
 
 
 def test_c2_small_forced_global(LA, orc):
