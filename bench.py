@@ -377,7 +377,12 @@ def main():
         "work": {"inserts": st["inserts"], "walk_steps": st["walk_steps"], "attempts": st["attempts"],
                  "ext_bases": st["ext_bases"], "ends_by_class": st["ends_by_class"],
                  "global_rounds": st["global_rounds"], "ends_medium": st["ends_medium"], "ends_xl": st["ends_xl"],
-                 "inserts_smem": st["inserts_smem"]},
+                 "inserts_smem": st["inserts_smem"],
+                 "classes": {n: {"ends": st["cls_ends"][i], "inserts": st["cls_inserts"][i],
+                                 "attempts": st["cls_attempts"][i], "filtered": st["cls_filtered"][i],
+                                 "ms": round(st["cls_ms"][i], 3)}
+                             for i, n in enumerate(["smem64x12", "smem128x6", "smem256x3", "smem256x2",
+                                                    "smem512x1", "xl512x1"])}},
         "roofline": roof,
         "roofline_hbm": {"bound": "hbm", "achieved": hbm_bytes / (ms_max / args.steps / 1e3) / 1e9,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s",

@@ -111,6 +111,12 @@ typedef struct {
     double ms_smem_medium;       /* device time of the XL + 1- and 2-CTA/SM classes (in ms_smem)   */
     int64_t ends_xl;             /* ends whose table lived in the XL class's global scratch        */
     int64_t xl_scratch_bytes;
+    /* per table class: 0..4 shared memory (64, 128, 256@3, 256@2, 512 threads), 5 = XL */
+    int64_t cls_ends[6], cls_inserts[6], cls_attempts[6], cls_filtered[6];
+    double cls_ms[6];
+    /* LA_PROFILE=1 only: per class, summed clock64 cycles of the builders' leader (wait for the
+       walker, prefix, clear, filter pass, build pass, link) and of the walker (wait, walk) */
+    uint64_t prof_cycles[6][8];
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);

@@ -47,7 +47,10 @@ class la_stats(ctypes.Structure):
                 ("smem_bytes_per_cta", ctypes.c_int64), ("smem_ctas_per_sm", ctypes.c_int32),
                 ("global_rounds", ctypes.c_int32), ("ends_medium", ctypes.c_int64),
                 ("ms_smem_medium", ctypes.c_double), ("ends_xl", ctypes.c_int64),
-                ("xl_scratch_bytes", ctypes.c_int64)]
+                ("xl_scratch_bytes", ctypes.c_int64), ("cls_ends", ctypes.c_int64 * 6),
+                ("cls_inserts", ctypes.c_int64 * 6), ("cls_attempts", ctypes.c_int64 * 6),
+                ("cls_filtered", ctypes.c_int64 * 6), ("cls_ms", ctypes.c_double * 6),
+                ("prof_cycles", (ctypes.c_uint64 * 8) * 6)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_get_stats",

@@ -120,7 +120,10 @@ class LocalAssembler:
         s = L.la_stats()
         self._check(self._lib.la_get_stats(self._ctx, ctypes.byref(s)))
         d = {f: getattr(s, f) for f, _ in L.la_stats._fields_}
-        d["ends_by_class"] = list(s.ends_by_class)
+        for f, t in L.la_stats._fields_:
+            if hasattr(t, "_length_"):
+                v = getattr(s, f)
+                d[f] = [list(x) if hasattr(x, "_length_") else x for x in v]
         return d
 
     def close(self):

@@ -27,44 +27,49 @@ struct DevParams {
 
 __host__ __device__ __forceinline__ int kwords(int k) { return (2 * k + 63) >> 6; }
 
-struct Kmer {
-    uint64_t w[MAX_KW];
+// A k-mer with at most NW words (NW = 2 covers k <= 64: the inline-key path keeps half the registers).
+template <int NW>
+struct KmerN {
+    uint64_t w[NW];
 };
+using Kmer = KmerN<MAX_KW>;
 
 __device__ __forceinline__ uint64_t funnel64(uint64_t hi, uint64_t lo, int s) {
     return s ? ((hi << s) | (lo >> (64 - s))) : hi;
 }
 
 // k-mer of length k starting at base p of the packed sequence R (words in any address space).
-template <typename P>
-__device__ __forceinline__ Kmer extract_kmer(const P *R, int p, int k, int KW) {
-    Kmer K;
+template <int NW = MAX_KW, typename P>
+__device__ __forceinline__ KmerN<NW> extract_kmer(const P *R, int p, int k, int KW) {
+    KmerN<NW> K;
     const int q = p >> 5, s = (p & 31) << 1;
 #pragma unroll
-    for (int w = 0; w < MAX_KW; ++w) {
+    for (int w = 0; w < NW; ++w) {
         if (w < KW) K.w[w] = funnel64(R[q + w], R[q + w + 1], s);
         else K.w[w] = 0;
     }
     const int pad = 64 * KW - 2 * k;
 #pragma unroll
-    for (int w = 0; w < MAX_KW; ++w)
+    for (int w = 0; w < NW; ++w)
         if (w == KW - 1 && pad) K.w[w] &= (~0ull) << pad;
     return K;
 }
 
 // next_kmer (Alg 2 line 15): drop base 0, append base b.
-__device__ __forceinline__ void roll_kmer(Kmer &K, int k, int KW, uint32_t b) {
+template <int NW>
+__device__ __forceinline__ void roll_kmer(KmerN<NW> &K, int k, int KW, uint32_t b) {
 #pragma unroll
-    for (int w = 0; w < MAX_KW; ++w) {
+    for (int w = 0; w < NW; ++w) {
         if (w < KW - 1) K.w[w] = (K.w[w] << 2) | (K.w[w + 1] >> 62);
         else if (w == KW - 1) K.w[w] = (K.w[w] << 2) | ((uint64_t)b << (64 * KW - 2 * k));
     }
 }
 
-__device__ __forceinline__ bool kmer_eq(const Kmer &a, const Kmer &b, int KW) {
+template <int NW>
+__device__ __forceinline__ bool kmer_eq(const KmerN<NW> &a, const KmerN<NW> &b, int KW) {
     bool eq = true;
 #pragma unroll
-    for (int w = 0; w < MAX_KW; ++w)
+    for (int w = 0; w < NW; ++w)
         if (w < KW) eq &= (a.w[w] == b.w[w]);
     return eq;
 }
@@ -80,10 +85,23 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
 
 // Hash of a k-mer: polynomial combine of the words + murmur3 fmix64.  The hash function does not
 // affect results (reading #17), only probe lengths and filter false positives.
-__device__ __forceinline__ uint64_t hash_kmer(const Kmer &K, int KW) {
+template <int NW>
+__device__ __forceinline__ uint64_t hash_kmer(const KmerN<NW> &K, int KW) {
+    if (NW <= 2) {
+        // k <= 64: a 32-bit multiply-xorshift mix of the four 32-bit halves (fewer instructions than
+        // 64-bit arithmetic); the high word (filter index, tag) is a second multiplicative mix.
+        const uint64_t w1 = (NW > 1 && KW > 1) ? K.w[NW > 1 ? 1 : 0] : 0ull;
+        uint32_t h = ((uint32_t)K.w[0] ^ ((uint32_t)(K.w[0] >> 32) * 0x85EBCA6Bu)) * 0xCC9E2D51u;
+        h ^= ((uint32_t)w1 ^ ((uint32_t)(w1 >> 32) * 0x27D4EB2Fu)) * 0x1B873593u;
+        h ^= h >> 15;
+        h *= 0x2C1B3C6Du;
+        h ^= h >> 12;
+        const uint32_t g = (h ^ (h >> 16)) * 0x9E3779B9u;
+        return ((uint64_t)(g | 1u) << 32) | h;
+    }
     uint64_t h = K.w[0];
 #pragma unroll
-    for (int w = 1; w < MAX_KW; ++w)
+    for (int w = 1; w < NW; ++w)
         if (w < KW) h = h * 0x9E3779B97F4A7C15ull + K.w[w];
     h ^= h >> 33;
     h *= 0xff51afd7ed558ccdull;

@@ -38,24 +38,38 @@ __host__ __device__ __forceinline__ uint32_t key_bytes(int k) { return inline_ke
 struct SmemFixed {
     uint32_t icap;        // slots an info buffer can describe (max table capacity)
     uint32_t off_info1, off_walk, off_tab, tab_bytes;
+    uint32_t off_filt, filt_bytes;   // XL only: the filter bitmaps stay in shared memory
 };
 
-// gt_stride > 0: the table region lives in a per-CTA global-memory scratch of gt_stride bytes (XL
-// class); shared memory then holds only the two info buffers and the walk strings.
+constexpr uint32_t XL_ICAP = 16384u;   // XL: info buffers of 64 KB each; the rest of smem = filter
+
+// gt_stride > 0: the table lives in a per-CTA global-memory scratch of gt_stride bytes (XL class);
+// shared memory then holds the two info buffers, the walk strings and the filter bitmaps.
 __host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, uint32_t gt_stride = 0) {
     SmemFixed F;
     const uint32_t Wp = ((uint32_t)W + 15u) & ~15u;
     const uint32_t fixed = 4u * Wp + 128u;
     const uint32_t rem = bytes > fixed ? bytes - fixed : 0u;
-    F.icap = (gt_stride ? rem / 8u : rem / 32u) & ~3u;   // (24 B inline slot +) 2 x 4 B info
+    if (gt_stride) {
+        F.icap = rem / 16u;   // at most half of shared memory for the info buffers
+        if (F.icap > XL_ICAP) F.icap = XL_ICAP;
+        F.icap &= ~3u;
+    } else {
+        F.icap = (rem / 32u) & ~3u;   // 24 B inline slot + 2 x 4 B info
+    }
     F.off_info1 = F.icap * 4u;
     F.off_walk = F.off_info1 + F.icap * 4u;
+    const uint32_t after = (F.off_walk + 4u * Wp + 15u) & ~15u;
     if (gt_stride) {
         F.off_tab = 0u;   // relative to the CTA's global scratch
         F.tab_bytes = gt_stride;
+        F.off_filt = after;
+        F.filt_bytes = bytes > after + 32u ? ((bytes - after - 32u) & ~31u) : 0u;
     } else {
-        F.off_tab = (F.off_walk + 4u * Wp + 15u) & ~15u;
+        F.off_tab = after;
         F.tab_bytes = bytes > F.off_tab + 32u ? bytes - F.off_tab - 32u : 0u;
+        F.off_filt = 0u;
+        F.filt_bytes = 0u;
     }
     return F;
 }
@@ -65,36 +79,60 @@ struct SmemTab {
 };
 
 __host__ __device__ __forceinline__ uint32_t pref_bytes(int r) { return (((uint32_t)r + 1u) * 4u + 15u) & ~15u; }
+// shared-memory copy of the end's reads: packed bases + quality classes (SW words each), u16 length,
+// u8 has-N flag
+__host__ __device__ __forceinline__ uint32_t stage_bytes(int r, int SW) {
+    return (((uint32_t)r * (uint32_t)SW * 16u + (uint32_t)r * 3u) + 15u) & ~15u;
+}
 
 // U = voting-occurrence upper bound (sum over reads of max(0, len-k)); the table region starts with
 // the per-read position prefix array (pref_bytes(r)).
+// Counters: shared-memory tables pack lo[4] | hi[4] as 8-bit fields (8 B, carry detected); global
+// (XL) tables use 8 x u32 (32 B) updated with fire-and-forget RED.ADD.
+__host__ __device__ __forceinline__ uint32_t cnt_bytes(bool gt) { return gt ? 32u : 8u; }
+
 __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_t U, bool allow_filter,
-                                                     uint32_t kbytes, int r) {
+                                                     uint32_t kbytes, int r, bool gt, int SW) {
     SmemTab T;
-    const uint32_t pb = pref_bytes(r);
+    const uint32_t sb = gt ? 0u : stage_bytes(r, SW);   // shared-memory tables: reads staged first
+    const uint32_t pb = pref_bytes(r) + sb;
     const uint32_t tab = F.tab_bytes > pb ? F.tab_bytes - pb : 0u;
-    const uint32_t per_slot = kbytes + 8u;
+    const uint32_t per_slot = kbytes + cnt_bytes(gt);
     uint32_t cap_nf = tab / per_slot;
     if (cap_nf > F.icap) cap_nf = F.icap;
     cap_nf &= ~1u;
     uint32_t mwords = 0, cap = cap_nf;
-    if (allow_filter && (float)U > SMEM_MAX_LOAD * (float)cap_nf) {
-        // two bitmaps of ~4 bits per occurrence each, at most a quarter of the region each
-        mwords = (4u * U + 31u) / 32u;
-        const uint32_t maxw = tab / 16u;
-        if (mwords > maxw) mwords = maxw;
-        mwords = (mwords + 3u) & ~3u;
-        const uint32_t rem = tab > 8u * mwords + 16u ? tab - 8u * mwords - 16u : 0u;
-        cap = rem / per_slot;
-        if (cap > F.icap) cap = F.icap;
-        cap &= ~1u;
+    const bool filt = allow_filter && (float)U > SMEM_MAX_LOAD * (float)cap_nf;
+    if (gt) {   // filter in shared memory, table (after the prefix array) in the global scratch
+        if (filt) {
+            mwords = (4u * U + 31u) / 32u;
+            const uint32_t maxw = F.filt_bytes / 8u;
+            if (mwords > maxw) mwords = maxw;
+            mwords &= ~3u;
+        }
+        T.off_pref = 0u;
+        T.off_b1 = F.off_filt;
+        T.off_b2 = T.off_b1 + mwords * 4u;
+        T.off_keys = pb;
+    } else {
+        if (filt) {
+            // two bitmaps of ~4 bits per occurrence each, at most a quarter of the region each
+            mwords = (4u * U + 31u) / 32u;
+            const uint32_t maxw = tab / 16u;
+            if (mwords > maxw) mwords = maxw;
+            mwords = (mwords + 3u) & ~3u;
+            const uint32_t rem = tab > 8u * mwords + 16u ? tab - 8u * mwords - 16u : 0u;
+            cap = rem / per_slot;
+            if (cap > F.icap) cap = F.icap;
+            cap &= ~1u;
+        }
+        T.off_pref = F.off_tab + sb;
+        T.off_b1 = F.off_tab + pb;
+        T.off_b2 = T.off_b1 + mwords * 4u;
+        T.off_keys = (T.off_b2 + mwords * 4u + 15u) & ~15u;
     }
     T.cap = cap;
     T.mwords = mwords;
-    T.off_pref = F.off_tab;
-    T.off_b1 = F.off_tab + pb;
-    T.off_b2 = T.off_b1 + mwords * 4u;
-    T.off_keys = (T.off_b2 + mwords * 4u + 15u) & ~15u;
     T.off_cnts = T.off_keys + cap * kbytes;
     return T;
 }
@@ -107,12 +145,13 @@ __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
     return r < 50 ? 0.30f : (r < 200 ? 0.16f : 0.10f);
 }
 
-__device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t min_cap) {
+__device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t min_cap,
+                                     int SW) {
     if (bytes == 0) return false;
     const SmemFixed F = smem_fixed(P.W, bytes);
     if (F.tab_bytes == 0) return false;
     if (r > 16384) return false;
-    const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r);
+    const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r, false, SW);
     if (T.cap < min_cap) return false;
     if (T.mwords == 0) return true;   // U <= 0.7 cap: cannot overflow
     return filtered_fraction(r) * (float)U + 64.f <= SMEM_MAX_LOAD * (float)T.cap;
@@ -141,12 +180,12 @@ __host__ __device__ __forceinline__ uint32_t xl_needed_cap(int64_t r, int64_t U,
 __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_max, bool filter, uint32_t icap) {
     uint32_t cap = xl_needed_cap(r_max, U_max, filter);
     if (cap > icap) cap = icap;
-    const uint32_t mwords = filter ? (uint32_t)(((4 * U_max + 31) / 32 + 3) & ~3ll) : 0u;
-    return (pref_bytes((int)r_max) + 8u * mwords + 32u + cap * 24u + 255u) & ~255u;
+    return (pref_bytes((int)r_max) + 32u + cap * (16u + cnt_bytes(true)) + 255u) & ~255u;
 }
 
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
-                       const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, PlanBytes pb, uint32_t xl_bytes,
+                       const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW, PlanBytes pb,
+                       uint32_t xl_bytes,
                        int32_t *__restrict__ cls, int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
                        uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att, int32_t *__restrict__ lists,
                        uint32_t *__restrict__ keys, int32_t *__restrict__ list_G, int *__restrict__ ctr) {
@@ -165,7 +204,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         int sc = -1;
         if (U < (1ll << 30))
             for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
-                if (fits(r, U, P, pb.b[i], min_table_cap(pb.t[i]))) sc = i;
+                if (fits(r, U, P, pb.b[i], min_table_cap(pb.t[i]), SW)) sc = i;
         int64_t U0 = sumlen - r * (int64_t)P.k_start;   // LPT key: occurrences at k_start
         U0 = U0 < 0 ? 0 : (U0 > 0xffffffffll ? 0xffffffffll : U0);
         if (sc < 0 && xl_bytes && r <= 16384 && U <= XL_MAX_U &&
@@ -198,7 +237,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
 constexpr uint32_t NEXT_NONE = 0x0FFFFFFFu;   // info word: next slot (28 bits) << 4 | visited << 3 | code
 
 struct GlobalStats {
-    unsigned long long inserts, steps, attempts;
+    unsigned long long inserts, steps, attempts, filtered;   // filtered: attempts built with the filter
 };
 
 __device__ __forceinline__ uint32_t filt_index(uint64_t h, uint32_t mbits) {
@@ -241,7 +280,8 @@ __device__ __forceinline__ void ld128v(const uint64_t *p, uint64_t &x, uint64_t 
 
 // Stored form of an inline key: word 1 is complemented, so a real key never reads (0, 0) = empty
 // (k <= 63 leaves at least two zero pad bits in word 1).
-__device__ __forceinline__ void inline_form(const Kmer &K, int KW, uint64_t &a, uint64_t &b) {
+template <int NW>
+__device__ __forceinline__ void inline_form(const KmerN<NW> &K, int KW, uint64_t &a, uint64_t &b) {
     a = K.w[0];
     b = ~(KW >= 2 ? K.w[1] : 0ull);
 }
@@ -254,8 +294,8 @@ struct TabCtx {   // what a table operation needs
     int SW, k, KW;
 };
 
-template <bool INL>
-__device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const Kmer &K, uint64_t h) {
+template <bool INL, int NW>
+__device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> &K, uint64_t h) {
     uint32_t s = slot_of(h, T.cap);
     if (INL) {
         uint64_t a, b;
@@ -273,7 +313,7 @@ __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const Kmer &K, u
             const uint64_t w = T.keys[s];
             if (w == 0) return NONE;
             if ((w & TAG_MASK) == tag) {
-                const Kmer K2 = extract_kmer(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
+                const KmerN<NW> K2 = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
                 if (kmer_eq(K, K2, T.KW)) return s;
             }
             s = (s + 1 == T.cap) ? 0 : s + 1;
@@ -283,8 +323,8 @@ __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const Kmer &K, u
 }
 
 // Alg 1 line 5 (kmer_ht.insert) with the vote of the following base.
-template <bool INL, bool GT>
-__device__ __forceinline__ void tab_insert(const TabCtx &T, const Kmer &K, uint64_t h, uint32_t rid, int pos,
+template <bool INL, bool GT, int NW>
+__device__ __forceinline__ void tab_insert(const TabCtx &T, const KmerN<NW> &K, uint64_t h, uint32_t rid, int pos,
                                            uint32_t b, bool hi, int *nclaim, int claim_limit, volatile int *ovf) {
     uint32_t s = slot_of(h, T.cap);
     if (INL) {
@@ -324,24 +364,29 @@ __device__ __forceinline__ void tab_insert(const TabCtx &T, const Kmer &K, uint6
                 w = old;
             }
             if ((w & TAG_MASK) == tag) {
-                const Kmer K2 = extract_kmer(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
+                const KmerN<NW> K2 = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
                 if (kmer_eq(K, K2, T.KW)) break;
             }
             s = (s + 1 == T.cap) ? 0 : s + 1;
         }
     }
-    // 32-bit ATOMS.ADD (a 64-bit shared-memory add compiles to a CAS loop)
-    const uint32_t old = atomicAdd(&T.c32[2 * s], 1u << (8 * b));
-    if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit lo counter would carry
-    if (hi) atomicAdd(&T.c32[2 * s + 1], 1u << (8 * b));  // hi <= lo: cannot carry first
+    if (GT) {   // 8 x u32 in L2: RED.ADD, nothing to wait for
+        atomicAdd(&T.c32[8 * (size_t)s + b], 1u);
+        if (hi) atomicAdd(&T.c32[8 * (size_t)s + 4 + b], 1u);
+    } else {    // 32-bit ATOMS.ADD (a 64-bit shared-memory add compiles to a CAS loop)
+        const uint32_t old = atomicAdd(&T.c32[2 * s], 1u << (8 * b));
+        if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit lo counter would carry
+        if (hi) atomicAdd(&T.c32[2 * s + 1], 1u << (8 * b));  // hi <= lo: cannot carry first
+    }
 }
 
-// Every voting occurrence of the end's reads (streamed from global memory).  The end's positions with a
+// Every voting occurrence of the end's reads (staged in shared memory, or streamed from global memory
+// for the XL class: plain generic loads serve both).  The end's positions with a
 // following base are numbered 0..total-1 read by read (pref[j] = first number of read j); builder bt
 // takes the contiguous range [bt*total/NB, (bt+1)*total/NB), so work is balanced to one position and a
 // thread extracts a k-mer only where its range enters a read, then rolls it; the following base and
 // its quality class come from one 64-bit word per 32 positions.  f(K, rid, p, nb, hi) per vote.
-template <typename F>
+template <int NW, typename F>
 __device__ __forceinline__ void for_each_vote(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
                                               const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
                                               const uint32_t *pref, int64_t r0, int r, int SW, int k, int KW,
@@ -365,19 +410,19 @@ __device__ __forceinline__ void for_each_vote(const uint64_t *__restrict__ rseq,
         const int pe = min(npos, p + (int)(end - cur));
         const uint64_t *R = rseq + rid * SW;
         const uint64_t *Q = rqc + rid * SW;
-        Kmer K = extract_kmer(R, p, k, KW);
+        KmerN<NW> K = extract_kmer<NW>(R, p, k, KW);
         int lastN = -1;
-        if (__ldg(&rflag[rid]))   // this read has an N
+        if (rflag[rid])   // this read has an N
             for (int i = p; i < p + k; ++i)
                 if (get2(Q, i) == 3u) lastN = i;
         int wi = (p + k) >> 5;
-        uint64_t wR = __ldg(&R[wi]), wQ = __ldg(&Q[wi]);
+        uint64_t wR = R[wi], wQ = Q[wi];
         for (int q = p; q < pe; ++q) {
             const int i = q + k;
             if ((i >> 5) != wi) {
                 wi = i >> 5;
-                wR = __ldg(&R[wi]);
-                wQ = __ldg(&Q[wi]);
+                wR = R[wi];
+                wQ = Q[wi];
             }
             const int sh = 62 - ((i & 31) << 1);
             const uint32_t nb = (uint32_t)(wR >> sh) & 3u;
@@ -393,40 +438,229 @@ __device__ __forceinline__ void for_each_vote(const uint64_t *__restrict__ rseq,
     }
 }
 
-// ---- the kernel --------------------------------------------------------------------------------
-enum : int { ST_EMPTY = 0, ST_BUILD = 1, ST_WALK = 2 };
+// Batched variant for global-memory (XL) tables: positions are processed four at a time so that the
+// four hashes, filter probes and table probes are independent L2 requests in flight together.
+// f4(Kq, rid, p0, nbq, himask, vmask): bit u of vmask = position p0+u votes; of himask = high tier.
+template <int NW, int BATCH, typename F4>
+__device__ __forceinline__ void for_each_vote4(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+                                               const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
+                                               const uint32_t *pref, int64_t r0, int r, int SW, int k, int KW,
+                                               int bt, int NB, const volatile int *stop, F4 &&f4) {
+    const uint32_t total = pref[r];
+    uint32_t cur = (uint32_t)(((uint64_t)total * (uint32_t)bt) / (uint32_t)NB);
+    const uint32_t end = (uint32_t)(((uint64_t)total * (uint32_t)(bt + 1)) / (uint32_t)NB);
+    if (cur >= end) return;
+    int lo = 0, hi = r;
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (pref[mid] <= cur) lo = mid; else hi = mid;
+    }
+    int j = lo;
+    while (pref[j + 1] <= cur) ++j;
+    int p = (int)(cur - pref[j]);
+    while (cur < end) {
+        if (*stop) return;
+        const int64_t rid = r0 + j;
+        const int npos = (int)(pref[j + 1] - pref[j]);
+        const int pe = min(npos, p + (int)(end - cur));
+        const uint64_t *R = rseq + rid * SW;
+        const uint64_t *Q = rqc + rid * SW;
+        KmerN<NW> K = extract_kmer<NW>(R, p, k, KW);
+        int lastN = -1;
+        if (rflag[rid])
+            for (int i = p; i < p + k; ++i)
+                if (get2(Q, i) == 3u) lastN = i;
+        int wi = (p + k) >> 5;
+        uint64_t wR = R[wi], wQ = Q[wi];
+        for (int q = p; q < pe; q += BATCH) {
+            KmerN<NW> Kq[BATCH];
+            uint32_t nbq[BATCH];
+            uint32_t vm = 0, hm = 0;
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+                Kq[u] = K;
+                nbq[u] = 0;
+                const int qq = q + u;
+                if (qq < pe) {
+                    const int i = qq + k;
+                    if ((i >> 5) != wi) {
+                        wi = i >> 5;
+                        wR = R[wi];
+                        wQ = Q[wi];
+                    }
+                    const int sh = 62 - ((i & 31) << 1);
+                    const uint32_t nb = (uint32_t)(wR >> sh) & 3u;
+                    const uint32_t nq = (uint32_t)(wQ >> sh) & 3u;
+                    if (nq - 1u < 2u && lastN < qq) {
+                        vm |= 1u << u;
+                        if (nq == 2u) hm |= 1u << u;
+                    }
+                    if (nq == 3u) lastN = i;
+                    nbq[u] = nb;
+                    roll_kmer(K, k, KW, nb);
+                }
+            }
+            if (vm) f4(Kq, (uint32_t)rid, q, nbq, hm, vm);
+        }
+        cur += (uint32_t)(pe - p);
+        ++j;
+        p = 0;
+        while (cur < end && pref[j + 1] == pref[j]) ++j;
+    }
+}
 
+// Four inline-key inserts with interleaved probing: each round issues the probe loads of all pending
+// inserts before resolving any of them (s[u]: start slot of insert u).
+template <bool GT, int NW, int BATCH>
+__device__ __forceinline__ void tab_insert4_inline(const TabCtx &T, const KmerN<NW> (&Kq)[BATCH], uint32_t (&s)[BATCH],
+                                                   const uint32_t (&nbq)[BATCH], uint32_t hm, uint32_t pm, int *nclaim,
+                                                   int claim_limit, volatile int *ovf) {
+    while (pm) {
+        uint64_t x[BATCH], y[BATCH];
+#pragma unroll
+        for (int u = 0; u < BATCH; ++u)
+            if ((pm >> u) & 1u) ld128v<GT>(&T.keys[2 * (size_t)s[u]], x[u], y[u]);
+#pragma unroll
+        for (int u = 0; u < BATCH; ++u) {
+            if (!((pm >> u) & 1u)) continue;
+            uint64_t a, bb;
+            inline_form(Kq[u], T.KW, a, bb);
+            bool found = false;
+            if (y[u] == 0) {
+                if (*ovf) { pm &= ~(1u << u); continue; }
+                cas128<GT>((void *)&T.keys[2 * (size_t)s[u]], 0ull, 0ull, a, bb, x[u], y[u]);
+                if (y[u] == 0) {
+                    found = true;
+                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
+                }
+            } else if (y[u] == bb && x[u] != a) {
+                x[u] = *(volatile uint64_t *)&T.keys[2 * (size_t)s[u]];
+            }
+            if (found || (x[u] == a && y[u] == bb)) {
+                if (GT) {
+                    atomicAdd(&T.c32[8 * (size_t)s[u] + nbq[u]], 1u);
+                    if ((hm >> u) & 1u) atomicAdd(&T.c32[8 * (size_t)s[u] + 4 + nbq[u]], 1u);
+                } else {
+                    const uint32_t old = atomicAdd(&T.c32[2 * s[u]], 1u << (8 * nbq[u]));
+                    if (((old >> (8 * nbq[u])) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit counter would carry
+                    if ((hm >> u) & 1u) atomicAdd(&T.c32[2 * s[u] + 1], 1u << (8 * nbq[u]));
+                }
+                pm &= ~(1u << u);
+            } else {
+                s[u] = (s[u] + 1 == T.cap) ? 0 : s[u] + 1;
+            }
+        }
+    }
+}
+
+// ---- the kernel --------------------------------------------------------------------------------
 struct EndSlot {            // one contig end in flight
-    int e, r;
+    int e, r, ulen;         // ulen: common length of all the end's reads (0 if they differ)
     long long r0;
     int k, shift, kmax_eff, attempts;
     int best_len, best_term, best_k, best_buf;
-    int status;             // ST_*; written after a fence, polled with volatile loads
+    int done, dead, ovf;    // done: finished (refill); dead: no more ends; ovf: redo in the global path
     uint32_t start;         // the start k-mer's slot (NONE if absent) of the last build
     unsigned long long ins, steps;
 };
 
 struct BuildCtl {           // builders' shared scratch
-    int slot;               // end slot chosen by the builders' leader (-1: exit)
+    int skip;               // 1: the current slot has no work (retired)
     int overflow, nclaim;
     uint32_t start;
+    int lmin, lmax;
     uint32_t wsum[16];      // per builder warp: prefix-scan totals
 };
 
 __device__ __forceinline__ void builders_sync(int NB) { asm volatile("bar.sync 1, %0;" ::"r"(NB) : "memory"); }
+
+// mbarrier handoff between the builders' leader and the walker (hardware-suspended waits).
+__device__ __forceinline__ uint32_t smem_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+// try_wait suspends for a hardware-chosen window; between failed tries the waiter sleeps so that a
+// long wait does not take issue slots from the builders on the same SM.
+__device__ __forceinline__ bool mbar_try_wait(uint32_t addr, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(addr), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    const uint32_t addr = smem_addr(bar);
+    while (!mbar_try_wait(addr, parity)) __nanosleep(200);
+}
 
 template <bool INL, bool GT>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
                                            const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
                                            const uint32_t *pref, long long r0, int r, const DevParams &P,
-                                           const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, int bt, int NB) {
+                                           const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, int bt, int NB,
+                                           long long &t_filter, long long &t_build) {
     const volatile int *stop = &B.overflow;
     const int k = T.k, KW = T.KW;
+    constexpr int NW = INL ? 2 : MAX_KW;   // inline keys: k <= 63 fits two words
+    constexpr int BATCH = GT ? 4 : 2;      // positions in flight per thread (register budget)
+    if (GT && INL) {   // global-memory table: batched passes (positions in flight hide L2 latency)
+        if (mbits) {
+            for_each_vote4<NW, BATCH>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
+                           [&](const KmerN<NW> (&Kq)[BATCH], uint32_t, int, const uint32_t (&)[BATCH], uint32_t, uint32_t vm) {
+                               uint32_t fi[BATCH], w2[BATCH], need = 0;
+#pragma unroll
+                               for (int u = 0; u < BATCH; ++u)
+                                   if ((vm >> u) & 1u) {
+                                       fi[u] = filt_index(hash_kmer(Kq[u], KW), mbits);
+                                       w2[u] = *(volatile uint32_t *)&B2[fi[u] >> 5];
+                                   }
+                               uint32_t old[BATCH];
+#pragma unroll
+                               for (int u = 0; u < BATCH; ++u)
+                                   if (((vm >> u) & 1u) && !((w2[u] >> (fi[u] & 31)) & 1u)) {
+                                       old[u] = atomicOr(&B1[fi[u] >> 5], 1u << (fi[u] & 31));
+                                       need |= 1u << u;
+                                   }
+#pragma unroll
+                               for (int u = 0; u < BATCH; ++u)
+                                   if (((need >> u) & 1u) && ((old[u] >> (fi[u] & 31)) & 1u))
+                                       atomicOr(&B2[fi[u] >> 5], 1u << (fi[u] & 31));
+                           });
+            builders_sync(NB);
+        }
+        t_filter = clock64();
+        const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
+        for_each_vote4<NW, BATCH>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
+                       [&](const KmerN<NW> (&Kq)[BATCH], uint32_t, int, const uint32_t (&nbq)[BATCH], uint32_t hm, uint32_t vm) {
+                           uint32_t sl[BATCH], w2[BATCH], fi[BATCH];
+                           uint32_t pm = vm;
+#pragma unroll
+                           for (int u = 0; u < BATCH; ++u) {
+                               const uint64_t h = hash_kmer(Kq[u], KW);
+                               sl[u] = slot_of(h, T.cap);
+                               fi[u] = filt_index(h, mbits);
+                           }
+                           if (mbits) {
+#pragma unroll
+                               for (int u = 0; u < BATCH; ++u)
+                                   if ((vm >> u) & 1u) w2[u] = B2[fi[u] >> 5];
+#pragma unroll
+                               for (int u = 0; u < BATCH; ++u)
+                                   if (((vm >> u) & 1u) && !((w2[u] >> (fi[u] & 31)) & 1u)) pm &= ~(1u << u);
+                           }
+                           if (pm) tab_insert4_inline<GT, NW, BATCH>(T, Kq, sl, nbq, hm, pm, &B.nclaim, claim_limit, &B.overflow);
+                       });
+    } else {
     // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
     if (mbits) {
-        for_each_vote(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const Kmer &K, uint32_t, int, uint32_t, bool) {
+        for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
+                      [&](const KmerN<NW> &K, uint32_t, int, uint32_t, bool) {
                           const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
                           const uint32_t bit = 1u << (fi & 31);
                           if (!(B2[fi >> 5] & bit)) {
@@ -436,45 +670,55 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                       });
         builders_sync(NB);
     }
+    t_filter = clock64();
     // ---- build (Alg 1) ----
     const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
-    for_each_vote(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const Kmer &K, uint32_t rid, int p, uint32_t nb, bool hi) {
+    for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
+                      [&](const KmerN<NW> &K, uint32_t rid, int p, uint32_t nb, bool hi) {
                           const uint64_t h = hash_kmer(K, KW);
                           if (mbits) {
                               const uint32_t fi = filt_index(h, mbits);
                               if (!((B2[fi >> 5] >> (fi & 31)) & 1u)) return;
                           }
-                          tab_insert<INL, GT>(T, K, h, rid, p, nb, hi, &B.nclaim, claim_limit, &B.overflow);
+                          tab_insert<INL, GT, NW>(T, K, h, rid, p, nb, hi, &B.nclaim, claim_limit, &B.overflow);
                       });
+    }
     builders_sync(NB);
+    t_build = clock64();
     if (B.overflow) return;
     // ---- ext rule + successor links (a5) into the end's info buffer ----
     for (uint32_t s = bt; s < T.cap; s += NB) {
-        Kmer K;
+        KmerN<NW> K;
         if (INL) {
             const ulonglong2 w = ((const ulonglong2 *)T.keys)[s];
             if (w.y == 0) continue;
+#pragma unroll
+            for (int i = 0; i < NW; ++i) K.w[i] = 0;
             K.w[0] = w.x;
-            K.w[1] = KW >= 2 ? ~w.y : 0ull;
-            K.w[2] = K.w[3] = 0;
+            if (NW > 1) K.w[NW > 1 ? 1 : 0] = KW >= 2 ? ~w.y : 0ull;
         } else {
             const uint64_t w = T.keys[s];
             if (w == 0) continue;
-            K = extract_kmer(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
+            K = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
         }
-        const uint32_t lw = T.c32[2 * s], hw = T.c32[2 * s + 1];
         uint32_t lo[4], hi[4];
+        if (GT) {
+            const uint4 a = ((const uint4 *)T.c32)[2 * (size_t)s], c = ((const uint4 *)T.c32)[2 * (size_t)s + 1];
+            lo[0] = a.x; lo[1] = a.y; lo[2] = a.z; lo[3] = a.w;
+            hi[0] = c.x; hi[1] = c.y; hi[2] = c.z; hi[3] = c.w;
+        } else {
+            const uint32_t lw = T.c32[2 * s], hw = T.c32[2 * s + 1];
 #pragma unroll
-        for (int b = 0; b < 4; ++b) {
-            lo[b] = (lw >> (8 * b)) & 0xffu;
-            hi[b] = (hw >> (8 * b)) & 0xffu;
+            for (int b = 0; b < 4; ++b) {
+                lo[b] = (lw >> (8 * b)) & 0xffu;
+                hi[b] = (hw >> (8 * b)) & 0xffu;
+            }
         }
         const int code = ext_rule(lo, hi, P.V, P.F);
         uint32_t nxt = NEXT_NONE;
         if (code < 4) {
             roll_kmer(K, k, KW, (uint32_t)code);
-            const uint32_t t = tab_lookup<INL>(T, K, hash_kmer(K, KW));
+            const uint32_t t = tab_lookup<INL, NW>(T, K, hash_kmer(K, KW));
             nxt = t == NONE ? NEXT_NONE : t;
         }
         info[s] = (nxt << 4) | (uint32_t)code;
@@ -489,8 +733,8 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             uint64_t Tw[TAIL_W];
 #pragma unroll
             for (int i = 0; i < TAIL_W; ++i) Tw[i] = tail_e[i];
-            const Kmer K = extract_kmer(Tw, p, k, KW);
-            st = tab_lookup<INL>(T, K, hash_kmer(K, KW));
+            const KmerN<NW> K = extract_kmer<NW>(Tw, p, k, KW);
+            st = tab_lookup<INL, NW>(T, K, hash_kmer(K, KW));
         }
         B.start = st;
     }
@@ -506,13 +750,13 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     uint32_t smem_bytes, uint8_t *__restrict__ walk_buf, int32_t *__restrict__ out_len,
     uint8_t *__restrict__ out_term, uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
     int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
-    unsigned char *__restrict__ gscratch, uint32_t gstride) {
+    unsigned char *__restrict__ gscratch, uint32_t gstride, unsigned long long *__restrict__ prof) {
     static_assert(BLOCK >= 64, "one walker warp + at least one builder warp");
     constexpr int NB = BLOCK - 32;   // builder threads
     extern __shared__ __align__(16) unsigned char sm[];
     __shared__ EndSlot S[2];
     __shared__ BuildCtl B;
-    __shared__ int builders_done;
+    __shared__ __align__(8) uint64_t built[2], walked[2];   // mbarriers: slot s built / walked
     const int tid = threadIdx.x;
     const SmemFixed FX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u);
     // table region: shared memory, or this CTA's slice of the global scratch (XL class)
@@ -520,34 +764,43 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     const int Wp = (P.W + 15) & ~15;
     uint8_t *wstr = sm + FX.off_walk;   // end slot s: buffers 2s, 2s+1 (current / best)
     if (tid == 0) {
-        S[0].status = ST_EMPTY;
-        S[1].status = ST_EMPTY;
-        builders_done = 0;
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&built[i], 1);
+            mbar_init(&walked[i], 1);
+            S[i].done = 1;   // empty: the builders fetch an end first
+            S[i].dead = 0;
+            S[i].ovf = 0;
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
 
+    // The two end slots strictly alternate: builders build slot 0, slot 1, then wait for slot 0's
+    // walk, rebuild it (next k) or refill it (next end), and so on; the walker walks 0, 1, 0, ...
     if (tid < 32) {
         // ============================ walker warp ============================
         const int lane = tid;
         unsigned long long acc_ins = 0, acc_steps = 0, acc_att = 0;
-        int pref = 0;
-        for (;;) {
-            int s = -1;
-            if (lane == 0) {
-                for (;;) {
-                    if (*(volatile int *)&S[pref].status == ST_WALK) { s = pref; break; }
-                    if (*(volatile int *)&S[pref ^ 1].status == ST_WALK) { s = pref ^ 1; break; }
-                    // builders finish only when both end slots are empty, so nothing is left to walk
-                    if (*(volatile int *)&builders_done) break;
-                    __nanosleep(32);
-                }
-                __threadfence_block();
-            }
-            s = __shfl_sync(0xffffffffu, s, 0);
-            if (s < 0) break;
-            pref = s ^ 1;
+        uint32_t phase = 0u, alive = 3u;   // bit s: mbarrier parity / slot still in use
+        long long w_wait = 0, w_walk = 0;
+        for (int s = 0; alive; s ^= 1) {
+            if (!((alive >> s) & 1u)) continue;
+            const long long tw0 = clock64();
+            if (lane == 0) mbar_wait(&built[s], (phase >> s) & 1u);
+            w_wait += clock64() - tw0;
+            phase ^= 1u << s;
+            __syncwarp();
             EndSlot &E = S[s];
+            if (E.dead) {
+                alive &= ~(1u << s);
+                continue;
+            }
+            if (E.ovf) {   // the build overflowed: the global path owns this end; pass the slot back
+                if (lane == 0) mbar_arrive(&walked[s]);
+                continue;
+            }
             int done = 0, bl = 0, bb = 0;
+            const long long tw1 = clock64();
             if (lane == 0) {
                 // ---- walk (Alg 2) over the successor links ----
                 uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
@@ -585,6 +838,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             done = __shfl_sync(0xffffffffu, done, 0);
             bl = __shfl_sync(0xffffffffu, bl, 0);
             bb = __shfl_sync(0xffffffffu, bb, 0);
+            w_walk += clock64() - tw1;
             if (done) {
                 // ---- the selected walk -> HBM ----
                 const int e = E.e;
@@ -599,112 +853,184 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                     acc_ins += E.ins;
                     acc_steps += E.steps;
                     acc_att += E.attempts;
+                    E.done = 1;
                 }
             }
             __syncwarp();
-            if (lane == 0) {
-                __threadfence_block();
-                *(volatile int *)&E.status = done ? ST_EMPTY : ST_BUILD;
-            }
+            if (lane == 0) mbar_arrive(&walked[s]);   // release: the state above is visible to the builders
         }
         if (lane == 0) {
             atomicAdd(&gstats->inserts, acc_ins);
             atomicAdd(&gstats->steps, acc_steps);
             atomicAdd(&gstats->attempts, acc_att);
+            if (prof) {
+                atomicAdd(&prof[6], (unsigned long long)w_wait);
+                atomicAdd(&prof[7], (unsigned long long)w_walk);
+            }
         }
         return;
     }
 
     // ============================ builders ============================
     const int bt = tid - 32;
-    int pref = 0;
-    bool no_more = false;
-    for (;;) {
+    uint32_t wphase = 0u, first = 3u, alive = 3u;   // bit s; alive is identical in every builder
+    unsigned long long n_filtered = 0;
+    long long b_t[6] = {0, 0, 0, 0, 0, 0};   // builder-leader cycles: wait, prefix, clear, filter, build, link
+    for (int s = 0; alive; s ^= 1) {
+        if (!((alive >> s) & 1u)) continue;
+        EndSlot &E = S[s];
+        const long long ta = clock64();
         if (bt == 0) {
-            int s = -1;
-            for (;;) {
-                for (int c = 0; c < 2 && s < 0; ++c) {
-                    const int cand = pref ^ c;
-                    const int st = *(volatile int *)&S[cand].status;
-                    if (st == ST_BUILD) {
-                        __threadfence_block();
-                        s = cand;
-                    } else if (st == ST_EMPTY && !no_more) {
-                        const int idx = atomicAdd(work_ctr, 1);
-                        if (idx >= n_list) { no_more = true; continue; }
-                        const int e = list[idx];
-                        EndSlot &E = S[cand];
-                        E.e = e;
-                        E.r0 = eoff[e];
-                        E.r = (int)(eoff[e + 1] - E.r0);
-                        E.kmax_eff = min(P.k_max, (int)clen[e]);
-                        E.k = P.k_start;
-                        E.shift = 0;
-                        E.attempts = 0;
-                        E.best_len = -1;
-                        E.best_term = T_DEADEND;
-                        E.best_k = 0;
-                        E.best_buf = 1;
-                        E.ins = 0;
-                        E.steps = 0;
-                        s = cand;
-                    }
-                }
-                if (s >= 0) break;
-                if (no_more && *(volatile int *)&S[0].status == ST_EMPTY && *(volatile int *)&S[1].status == ST_EMPTY)
-                    break;
-                __nanosleep(32);
+            if (!((first >> s) & 1u)) {
+                mbar_wait(&walked[s], (wphase >> s) & 1u);   // acquire: the walker's update of slot s
+                wphase ^= 1u << s;
             }
-            B.slot = s;
+            first &= ~(1u << s);
+            B.skip = 0;
             B.overflow = 0;
             B.nclaim = 0;
-            if (s >= 0) pref = s ^ 1;
+            if (E.done) {   // refill the slot with the next end, or retire it
+                const int idx = atomicAdd(work_ctr, 1);
+                if (idx >= n_list) {
+                    E.dead = 1;
+                    B.skip = 1;
+                    mbar_arrive(&built[s]);   // the walker sees `dead` and retires the slot too
+                } else {
+                    const int e = list[idx];
+                    E.e = e;
+                    E.r0 = eoff[e];
+                    E.r = (int)(eoff[e + 1] - E.r0);
+                    E.ulen = -1;   // unknown until the first prefix pass
+                    E.kmax_eff = min(P.k_max, (int)clen[e]);
+                    E.k = P.k_start;
+                    E.shift = 0;
+                    E.attempts = 0;
+                    E.best_len = -1;
+                    E.best_term = T_DEADEND;
+                    E.best_k = 0;
+                    E.best_buf = 1;
+                    E.ins = 0;
+                    E.steps = 0;
+                    E.done = 0;
+                    E.ovf = 0;
+                }
+            }
         }
         builders_sync(NB);
-        const int s = B.slot;
-        if (s < 0) break;
-        EndSlot &E = S[s];
+        const long long tb = clock64();
+        b_t[0] += tb - ta;
+        if (B.skip) {
+            alive &= ~(1u << s);
+            continue;
+        }
         const int k = E.k;
         const int KW = kwords(k);
         const bool INL = inline_keys(k);
         const long long r0 = E.r0;
         const int r = E.r;
+        const int ulen = E.ulen;
+        // shared-memory tables: stage the end's reads (coalesced 16 B copies); the XL class streams
+        // them from HBM/L2 instead
+        const uint64_t *gR = rseq, *gQ = rqc;
+        const uint16_t *gL = rlen;
+        const uint8_t *gF = rflag;
+        long long lr0 = r0;   // first read index in (gR, gQ, gL, gF)
+        unsigned char *stage = tbase + FX.off_tab;
+        const bool no_room = !GT && stage_bytes(r, SW) + pref_bytes(r) + 64u * 24u > FX.tab_bytes;
+        if (!GT && !no_room) {
+            uint64_t *sR = (uint64_t *)stage;
+            uint64_t *sQ = sR + (size_t)r * SW;
+            uint16_t *sL = (uint16_t *)(sQ + (size_t)r * SW);
+            uint8_t *sF = (uint8_t *)(sL + r);
+            const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
+            const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
+            const int n4 = r * SW / 2;   // SW is even
+            for (int i = bt; i < n4; i += NB) {
+                ((uint4 *)sR)[i] = __ldg(&a4[i]);
+                ((uint4 *)sQ)[i] = __ldg(&b4[i]);
+            }
+            for (int i = bt; i < r; i += NB) {
+                sL[i] = __ldg(&rlen[r0 + i]);
+                sF[i] = __ldg(&rflag[r0 + i]);
+            }
+            gR = sR;
+            gQ = sQ;
+            gL = sL;
+            gF = sF;
+            lr0 = 0;
+            builders_sync(NB);
+        }
         // positions with a following base, per read (exclusive prefix, pref[r] = U) -> table plan
-        uint32_t *pref = (uint32_t *)(tbase + FX.off_tab);
-        {
+        uint32_t *pref = (uint32_t *)(stage + (GT ? 0u : stage_bytes(r, SW)));
+        if (no_room) {   // the reads alone do not fit this CTA's shared memory: no table (overflow)
+        } else if (ulen >= 0) {   // all reads of the end have length ulen: arithmetic, no loads
+            const uint32_t np = (uint32_t)max(0, ulen - k);
+            for (int j = bt; j <= r; j += NB) pref[j] = (uint32_t)j * np;
+            builders_sync(NB);
+        } else {
             const int per = (r + NB - 1) / NB;
             const int j0 = min(r, bt * per), j1 = min(r, j0 + per);
             uint32_t loc = 0;
-            for (int j = j0; j < j1; ++j) loc += (uint32_t)max(0, (int)__ldg(&rlen[r0 + j]) - k);
+            int lmin = 1 << 30, lmax = -1;
+            for (int j = j0; j < j1; ++j) {
+                const int l = gL[lr0 + j];
+                loc += (uint32_t)max(0, l - k);
+                lmin = min(lmin, l);
+                lmax = max(lmax, l);
+            }
             const int lane = bt & 31, w = bt >> 5;
             uint32_t inc = loc;
             for (int o = 1; o < 32; o <<= 1) {
                 const uint32_t v = __shfl_up_sync(0xffffffffu, inc, o);
                 if (lane >= o) inc += v;
             }
+            for (int o = 16; o; o >>= 1) {
+                lmin = min(lmin, __shfl_xor_sync(0xffffffffu, lmin, o));
+                lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
+            }
+            if (bt == 0) {
+                B.lmin = 1 << 30;
+                B.lmax = -1;
+            }
             if (lane == 31) B.wsum[w] = inc;
             builders_sync(NB);
+            if (lane == 0) {
+                atomicMin(&B.lmin, lmin);
+                atomicMax(&B.lmax, lmax);
+            }
             uint32_t off = inc - loc;
             for (int i = 0; i < w; ++i) off += B.wsum[i];
             for (int j = j0; j < j1; ++j) {
                 pref[j] = off;
-                off += (uint32_t)max(0, (int)__ldg(&rlen[r0 + j]) - k);
+                off += (uint32_t)max(0, (int)gL[lr0 + j] - k);
             }
             if (bt == NB - 1) pref[r] = off;   // the last builder covers the last read (or none)
             builders_sync(NB);
+            if (bt == 0) E.ulen = (r > 0 && B.lmin == B.lmax) ? B.lmax : -2;   // -2: lengths differ
         }
-        const uint32_t U = pref[r];
-        const SmemTab TB = smem_tab(FX, U, P.V >= 2, key_bytes(k), r);
-        bool ovf = TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
+        const uint32_t U = no_room ? 0u : pref[r];
+        const long long tc = clock64();
+        b_t[1] += tc - tb;
+        long long td = tc, t_filter = tc, t_build = tc;
+        SmemTab TB = smem_tab(FX, U, P.V >= 2, key_bytes(k), r, GT, SW);
+        if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
+            const uint32_t need = xl_needed_cap(r, U, TB.mwords != 0);
+            if (TB.cap > need) {
+                TB.cap = (need + 1u) & ~1u;
+                TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
+            }
+        }
+        bool ovf = no_room || TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
         if (!ovf) {
             const uint32_t mbits = TB.mwords * 32u;
-            uint32_t *B1 = (uint32_t *)(tbase + TB.off_b1);
-            uint32_t *B2 = (uint32_t *)(tbase + TB.off_b2);
+            if (mbits) ++n_filtered;
+            uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);   // filters: always shared memory
+            uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
             TabCtx T;
             T.keys = (uint64_t *)(tbase + TB.off_keys);
             T.c32 = (uint32_t *)(tbase + TB.off_cnts);
             T.cap = TB.cap;
-            T.rseq = rseq;
+            T.rseq = gR;   // REF keys store read indices relative to gR
             T.SW = SW;
             T.k = k;
             T.KW = KW;
@@ -712,39 +1038,52 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             {
                 const uint4 z = make_uint4(0, 0, 0, 0);
                 uint4 *a = (uint4 *)T.keys;
-                const uint32_t n16 = (TB.cap * (key_bytes(k) + 8u)) / 16u;
+                const uint32_t n16 = (TB.cap * (key_bytes(k) + cnt_bytes(GT))) / 16u;
                 for (uint32_t i = bt; i < n16; i += NB) a[i] = z;
                 for (uint32_t i = bt; i < 2u * TB.mwords; i += NB) B1[i] = 0;   // B1, B2 contiguous
             }
             builders_sync(NB);
+            td = clock64();
+            t_filter = t_build = td;
             const int e = E.e;
             const int Tn = min((int)clen[e], 128);
             const uint64_t *tail_e = tail + (size_t)e * TAIL_W;
             const uint64_t n0 = tailN[2 * (size_t)e], n1 = tailN[2 * (size_t)e + 1];
             uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
             if (INL)
-                build_link<true, GT>(B, T, B1, B2, mbits, info, rqc, rlen, rflag, pref, r0, r, P, tail_e, Tn, n0, n1, bt, NB);
+                build_link<true, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
+                                     t_filter, t_build);
             else
-                build_link<false, GT>(B, T, B1, B2, mbits, info, rqc, rlen, rflag, pref, r0, r, P, tail_e, Tn, n0, n1, bt, NB);
+                build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
+                                      t_filter, t_build);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
         }
         builders_sync(NB);   // info buffer complete; the table is free for the next build
+        {
+            const long long te = clock64();
+            b_t[2] += td - tc;
+            b_t[3] += t_filter - td;
+            b_t[4] += t_build - t_filter;
+            b_t[5] += te - t_build;
+        }
         if (bt == 0) {
-            if (ovf) {   // table or counter overflow: the global path redoes this end from scratch
+            if (ovf) {
+                // table or counter overflow: the global path redoes this end from scratch; the
+                // slot is refilled on its next turn (the walker only passes it through)
                 ovf_list[atomicAdd(n_ovf, 1)] = E.e;
-                __threadfence_block();
-                *(volatile int *)&E.status = ST_EMPTY;
+                E.ovf = 1;
+                E.done = 1;
             } else {
                 E.start = B.start;
                 E.ins += U;
-                __threadfence_block();
-                *(volatile int *)&E.status = ST_WALK;
             }
+            mbar_arrive(&built[s]);   // release: info buffer + slot state visible to the walker
         }
     }
     if (bt == 0) {
-        __threadfence_block();
-        *(volatile int *)&builders_done = 1;
+        atomicAdd(&gstats->filtered, n_filtered);
+        if (prof)
+            for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
     }
 }
 

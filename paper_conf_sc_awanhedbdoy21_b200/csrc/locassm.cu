@@ -73,10 +73,11 @@ struct la_ctx {
         smem_key2, glob_list, ctrs, ext_off, ext_seq, gstats, cub_tmp;
     DevBuf g_state, g_act, g_act2, g_still, g_cap, g_nrd, g_capoff, g_rdoff, g_slots, g_cnt, g_vis,
         g_cur;
-    DevBuf lens64, xl_scratch;
+    DevBuf lens64, xl_scratch, prof;
     HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
     int64_t g_attempts = 0;
     cudaEvent_t ev[6] = {};
+    cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] start of XL
     la_stats stats{};
 };
 
@@ -174,6 +175,21 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     cudaDeviceProp prop;
     cudaGetDeviceProperties(&prop, device);
     ctx->n_sm = prop.multiProcessorCount;
+    // tuning hook: LA_CLASSES="64x12,128x6,256x3,256x2,512x1" (threads x CTAs/SM per class)
+    if (const char *cfg = getenv("LA_CLASSES")) {
+        int t, c, n = 0;
+        const char *q = cfg;
+        while (n < N_SMEM_CLASSES && sscanf(q, "%dx%d", &t, &c) == 2) {
+            if (t == 64 || t == 96 || t == 128 || t == 192 || t == 256 || t == 512) {
+                ctx->cls_threads[n] = t;
+                ctx->cls_ctas[n] = std::max(1, c);
+            }
+            ++n;
+            q = strchr(q, ',');
+            if (!q) break;
+            ++q;
+        }
+    }
     // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
     for (int i = 0; i < N_SMEM_CLASSES; ++i) {
         size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - 512 /* static */;
@@ -189,11 +205,20 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
-    if (cudaFuncSetAttribute(k_smem<64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[0]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[1]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[3]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess ||
-        cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[4]) != cudaSuccess) {
+    for (auto &e : ctx->ev_cls) cudaEventCreate(&e);
+    bool attr_ok = cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        ctx->cls_bytes[N_SMEM_CLASSES - 1]) == cudaSuccess;
+    {
+        uint32_t mx = 0;
+        for (int i = 0; i < N_SMEM_CLASSES; ++i) mx = std::max(mx, ctx->cls_bytes[i]);
+        attr_ok &= cudaFuncSetAttribute(k_smem<64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<96, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<192, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+    }
+    if (!attr_ok) {
         cudaGetLastError();
         la_destroy(ctx);
         return LA_ERR_CUDA;
@@ -214,11 +239,13 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
                       &ctx->glob_list, &ctx->ctrs, &ctx->ext_off, &ctx->ext_seq, &ctx->gstats,
                       &ctx->cub_tmp, &ctx->g_state, &ctx->g_act, &ctx->g_act2, &ctx->g_still, &ctx->g_cap,
                       &ctx->g_nrd, &ctx->g_capoff, &ctx->g_rdoff, &ctx->g_slots, &ctx->g_cnt, &ctx->g_vis,
-                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch})
+                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch, &ctx->prof})
         b->release();
     for (HostBuf *b : {&ctx->h_ext_off, &ctx->h_ext_seq, &ctx->h_term, &ctx->h_k, &ctx->h_att, &ctx->h_small})
         b->release();
     for (auto &e : ctx->ev)
+        if (e) cudaEventDestroy(e);
+    for (auto &e : ctx->ev_cls)
         if (e) cudaEventDestroy(e);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
     delete ctx;
@@ -503,15 +530,15 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
     CK(grow(ctx->ctrs, 256));
-    CK(grow(ctx->gstats, 64));
+    CK(grow(ctx->gstats, 512));
     CK(grow(ctx->ext_off, (nE + 1) * 8));
-    CK(grow_host(ctx->h_small, 256));
+    CK(grow_host(ctx->h_small, 1024));
     int *d_ctr = P<int>(ctx->ctrs);   // [0..4] n per class [5] n_G [6] NOREADS [7] SHORT [15] n_ovf [16..20] work
     unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
 
     CK(cudaEventRecord(ctx->ev[0], st));
     CK(cudaMemsetAsync(d_ctr, 0, 128, st));
-    CK(cudaMemsetAsync(d_gst, 0, 64, st));
+    CK(cudaMemsetAsync(d_gst, 0, 512, st));
     int *h = (int *)ctx->h_small.p;
     int ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
     int n_glob = 0, n_xl = 0, xl_umax = 0, xl_rmax = 0;
@@ -529,7 +556,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         }
         if (force_smem) pb.b[0] = 0xffffffffu;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
-            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, pb,
+            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
             (force_global || force_smem) ? 0u : ctx->cls_bytes[N_SMEM_CLASSES - 1], P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
             lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
@@ -563,6 +590,14 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
     // XL (global-scratch tables) first, then the shared-memory classes from the largest tables
     // (1 CTA/SM, all shared memory) to the smallest (12 CTAs/SM)
+    // LA_PROFILE=1: per-class phase cycle counters (clock64) of the shared-memory kernels
+    unsigned long long *prof = nullptr;
+    if (getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE"))) {
+        CK(grow(ctx->prof, 8 * 8 * (N_SMEM_CLASSES + 1)));
+        prof = P<unsigned long long>(ctx->prof);
+        CK(cudaMemsetAsync(prof, 0, 8 * 8 * (N_SMEM_CLASSES + 1), st));
+    }
+    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES + 1], st));
     if (n_xl > 0) {
         const uint32_t bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
         const uint32_t icap = smem_fixed(dp.W, bytes, 1u).icap;
@@ -574,12 +609,13 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
             lst, n_xl, d_ctr + 21, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
             P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
             P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst, P<unsigned char>(ctx->xl_scratch),
-            stride);
+            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)(d_gst + 8 + 4 * N_SMEM_CLASSES),
+            P<unsigned char>(ctx->xl_scratch), stride, prof ? prof + 8 * N_SMEM_CLASSES : nullptr);
         CKL();
         ctx->stats.ends_xl = n_xl;
         ctx->stats.xl_scratch_bytes = (int64_t)grid * stride;
     }
+    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES], st));   // end of XL
     for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
         const int n = ncls[c];
         if (n > 0) {
@@ -593,9 +629,12 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
                                       P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                 \
                                       P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                       \
                                       P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                         \
-                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)d_gst, nullptr, 0u)
+                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,                          \
+                                      (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr)
             switch (ctx->cls_threads[c]) {
                 case 64: LA_LAUNCH_SMEM(64); break;
+                case 96: LA_LAUNCH_SMEM(96); break;
+                case 192: LA_LAUNCH_SMEM(192); break;
                 case 128: LA_LAUNCH_SMEM(128); break;
                 case 256: LA_LAUNCH_SMEM(256); break;
                 default: LA_LAUNCH_SMEM(512); break;
@@ -604,6 +643,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
             CKL();
         }
         if (c == 2) CK(cudaEventRecord(ctx->ev[5], st));   // after the 1- and 2-CTA/SM classes
+        CK(cudaEventRecord(ctx->ev_cls[c], st));   // end of class c
     }
     int n_ovf = 0;
     int n_smem = n_xl;
@@ -633,8 +673,22 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     int64_t *h64 = (int64_t *)ctx->h_small.p;
     CK(cudaMemcpyAsync(h64, P<int64_t>(ctx->ext_off) + nE, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(h64 + 1, d_gst, 40, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64 + 1, d_gst, 8 * (8 + 4 * (N_SMEM_CLASSES + 1)), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
+    if (prof) {
+        CK(cudaMemcpy(ctx->stats.prof_cycles, prof, sizeof(ctx->stats.prof_cycles), cudaMemcpyDeviceToHost));
+    }
+    // per-class stats (classes 0..4 shared memory, 5 = XL); fold them into the smem totals
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
+        const int64_t *g = h64 + 1 + 8 + 4 * c;
+        ctx->stats.cls_ends[c] = c < N_SMEM_CLASSES ? ncls[c] : n_xl;
+        ctx->stats.cls_inserts[c] = g[0];
+        ctx->stats.cls_attempts[c] = g[2];
+        ctx->stats.cls_filtered[c] = g[3];
+        h64[1] += g[0];
+        h64[2] += g[1];
+        h64[3] += g[2];
+    }
     const int64_t total = h64[0];
     // d_gst: [0] smem inserts [1] smem walk steps [2] smem attempts [3] global inserts [4] global steps
     ctx->stats.inserts = h64[1] + h64[4];
@@ -685,6 +739,18 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     ctx->stats.ms_global = ms;
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
     ctx->stats.ms_emit = ms;
+    {
+        cudaEvent_t prev = ctx->ev_cls[N_SMEM_CLASSES + 1];
+        float m = 0;
+        cudaEventElapsedTime(&m, prev, ctx->ev_cls[N_SMEM_CLASSES]);
+        ctx->stats.cls_ms[N_SMEM_CLASSES] = m;
+        prev = ctx->ev_cls[N_SMEM_CLASSES];
+        for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
+            cudaEventElapsedTime(&m, prev, ctx->ev_cls[c]);
+            ctx->stats.cls_ms[c] = m;
+            prev = ctx->ev_cls[c];
+        }
+    }
     // class counts (host-side tally from the plan counters)
     ctx->stats.ends_by_class[2] = n_smem - n_ovf;
     ctx->stats.ends_by_class[3] = n_glob;
