@@ -22,7 +22,7 @@ FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std
 def build(force: bool = False, verbose: bool = False) -> str:
     stale = not os.path.exists(SO) or os.path.getmtime(SO) < max(os.path.getmtime(p) for p in DEPS)
     if force or stale:
-        cmd = [NVCC, *FLAGS, "-o", SO, *SRC]
+        cmd = [NVCC, *FLAGS, *os.environ.get("LA_NVCC_EXTRA", "").split(), "-o", SO, *SRC]
         if verbose:
             cmd.insert(1, "-Xptxas=-v")
             print(" ".join(cmd), file=sys.stderr)

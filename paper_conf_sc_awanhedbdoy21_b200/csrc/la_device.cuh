@@ -39,29 +39,31 @@ __device__ __forceinline__ uint64_t funnel64(uint64_t hi, uint64_t lo, int s) {
 }
 
 // k-mer of length k starting at base p of the packed sequence R (words in any address space).
+// Written with per-word selects only (no "if (w == KW - 1)" updates): that form lets the compiler turn
+// the unrolled loop into one dynamically indexed store, which puts the k-mer in local memory.
 template <int NW = MAX_KW, typename P>
 __device__ __forceinline__ KmerN<NW> extract_kmer(const P *R, int p, int k, int KW) {
     KmerN<NW> K;
     const int q = p >> 5, s = (p & 31) << 1;
 #pragma unroll
     for (int w = 0; w < NW; ++w) {
-        if (w < KW) K.w[w] = funnel64(R[q + w], R[q + w + 1], s);
-        else K.w[w] = 0;
+        const int bits = 2 * k - 64 * w;   // bits of word w that belong to the k-mer (> 0 iff w < KW)
+        const uint64_t m = bits >= 64 ? ~0ull : (~0ull << (64 - bits));
+        K.w[w] = w < KW ? (funnel64(R[q + w], R[q + w + 1], s) & m) : 0ull;
     }
-    const int pad = 64 * KW - 2 * k;
-#pragma unroll
-    for (int w = 0; w < NW; ++w)
-        if (w == KW - 1 && pad) K.w[w] &= (~0ull) << pad;
     return K;
 }
 
-// next_kmer (Alg 2 line 15): drop base 0, append base b.
+// next_kmer (Alg 2 line 15): drop base 0, append base b (the new base k-1 lands in word (k-1)/32).
 template <int NW>
 __device__ __forceinline__ void roll_kmer(KmerN<NW> &K, int k, int KW, uint32_t b) {
+    (void)KW;
+    const int wl = (k - 1) >> 5;
+    const uint64_t nb = ((uint64_t)b * 0x5555555555555555ull) & (3ull << (62 - 2 * ((k - 1) & 31)));
 #pragma unroll
     for (int w = 0; w < NW; ++w) {
-        if (w < KW - 1) K.w[w] = (K.w[w] << 2) | (K.w[w + 1] >> 62);
-        else if (w == KW - 1) K.w[w] = (K.w[w] << 2) | ((uint64_t)b << (64 * KW - 2 * k));
+        const uint64_t carry = (w + 1 < NW) ? (K.w[(w + 1 < NW) ? w + 1 : w] >> 62) : 0ull;
+        K.w[w] = (K.w[w] << 2) | carry | (w == wl ? nb : 0ull);
     }
 }
 

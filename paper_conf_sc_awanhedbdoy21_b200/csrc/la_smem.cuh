@@ -45,21 +45,24 @@ constexpr uint32_t XL_ICAP = 16384u;   // XL: info buffers of 64 KB each; the re
 
 // gt_stride > 0: the table lives in a per-CTA global-memory scratch of gt_stride bytes (XL class);
 // shared memory then holds the two info buffers, the walk strings and the filter bitmaps.
-__host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, uint32_t gt_stride = 0) {
+// single = true: one end in flight (k_small): one info buffer and two walk strings.
+__host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, uint32_t gt_stride = 0,
+                                                         bool single = false) {
     SmemFixed F;
     const uint32_t Wp = ((uint32_t)W + 15u) & ~15u;
-    const uint32_t fixed = 4u * Wp + 128u;
+    const uint32_t nwalk = single ? 2u : 4u;
+    const uint32_t fixed = nwalk * Wp + 128u;
     const uint32_t rem = bytes > fixed ? bytes - fixed : 0u;
     if (gt_stride) {
         F.icap = rem / 16u;   // at most half of shared memory for the info buffers
         if (F.icap > XL_ICAP) F.icap = XL_ICAP;
         F.icap &= ~3u;
     } else {
-        F.icap = (rem / 32u) & ~3u;   // 24 B inline slot + 2 x 4 B info
+        F.icap = (rem / (single ? 28u : 32u)) & ~3u;   // 24 B inline slot + 4 B info per end in flight
     }
-    F.off_info1 = F.icap * 4u;
-    F.off_walk = F.off_info1 + F.icap * 4u;
-    const uint32_t after = (F.off_walk + 4u * Wp + 15u) & ~15u;
+    F.off_info1 = single ? 0u : F.icap * 4u;
+    F.off_walk = (single ? 0u : F.off_info1) + F.icap * 4u;
+    const uint32_t after = (F.off_walk + nwalk * Wp + 15u) & ~15u;
     if (gt_stride) {
         F.off_tab = 0u;   // relative to the CTA's global scratch
         F.tab_bytes = gt_stride;
@@ -146,9 +149,9 @@ __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
 }
 
 __device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t min_cap,
-                                     int SW) {
+                                     int SW, bool single) {
     if (bytes == 0) return false;
-    const SmemFixed F = smem_fixed(P.W, bytes);
+    const SmemFixed F = smem_fixed(P.W, bytes, 0u, single);
     if (F.tab_bytes == 0) return false;
     if (r > 16384) return false;
     const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r, false, SW);
@@ -164,6 +167,7 @@ constexpr int N_SMEM_CLASSES = 5;
 struct PlanBytes {
     uint32_t b[N_SMEM_CLASSES];   // dynamic shared memory per CTA
     uint32_t t[N_SMEM_CLASSES];   // threads per CTA
+    uint32_t single;              // bit i: class i runs k_small (one end per CTA, no walker warp)
 };
 
 __host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { return 4u * threads; }
@@ -204,7 +208,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         int sc = -1;
         if (U < (1ll << 30))
             for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
-                if (fits(r, U, P, pb.b[i], min_table_cap(pb.t[i]), SW)) sc = i;
+                if (fits(r, U, P, pb.b[i], min_table_cap(pb.t[i]), SW, (pb.single >> i) & 1u)) sc = i;
         int64_t U0 = sumlen - r * (int64_t)P.k_start;   // LPT key: occurrences at k_start
         U0 = U0 < 0 ? 0 : (U0 > 0xffffffffll ? 0xffffffffll : U0);
         if (sc < 0 && xl_bytes && r <= 16384 && U <= XL_MAX_U &&
@@ -582,20 +586,74 @@ __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
-// try_wait suspends for a hardware-chosen window; between failed tries the waiter sleeps so that a
-// long wait does not take issue slots from the builders on the same SM.
+// try_wait with a suspend-time hint: the waiting thread is suspended in hardware until the phase
+// completes (or the hint, 1 ms, expires), so a long wait takes no issue slots from the builders on
+// the same SM (ncu: a polling loop with __nanosleep was 44% of the kernel's executed instructions).
 __device__ __forceinline__ bool mbar_try_wait(uint32_t addr, uint32_t parity) {
     uint32_t ok;
     asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}"
         : "=r"(ok)
-        : "r"(addr), "r"(parity)
+        : "r"(addr), "r"(parity), "r"(1000000u)
         : "memory");
     return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     const uint32_t addr = smem_addr(bar);
-    while (!mbar_try_wait(addr, parity)) __nanosleep(200);
+    while (!mbar_try_wait(addr, parity)) {
+    }
+}
+
+// Positions with a following base, per read: exclusive prefix pref[0..r] (pref[r] = U).  All NB
+// builder threads call it; E.ulen records whether every read of the end has the same length (then the
+// prefix is arithmetic from the next attempt on).
+__device__ __forceinline__ void read_prefix(BuildCtl &B, EndSlot &E, uint32_t *pref, const uint16_t *gL, long long lr0,
+                                            int r, int k, int ulen, int bt, int NB) {
+    if (ulen >= 0) {   // all reads of the end have length ulen: arithmetic, no loads
+        const uint32_t np = (uint32_t)max(0, ulen - k);
+        for (int j = bt; j <= r; j += NB) pref[j] = (uint32_t)j * np;
+        builders_sync(NB);
+    } else {
+        const int per = (r + NB - 1) / NB;
+        const int j0 = min(r, bt * per), j1 = min(r, j0 + per);
+        uint32_t loc = 0;
+        int lmin = 1 << 30, lmax = -1;
+        for (int j = j0; j < j1; ++j) {
+            const int l = gL[lr0 + j];
+            loc += (uint32_t)max(0, l - k);
+            lmin = min(lmin, l);
+            lmax = max(lmax, l);
+        }
+        const int lane = bt & 31, w = bt >> 5;
+        uint32_t inc = loc;
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t v = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += v;
+        }
+        for (int o = 16; o; o >>= 1) {
+            lmin = min(lmin, __shfl_xor_sync(0xffffffffu, lmin, o));
+            lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
+        }
+        if (bt == 0) {
+            B.lmin = 1 << 30;
+            B.lmax = -1;
+        }
+        if (lane == 31) B.wsum[w] = inc;
+        builders_sync(NB);
+        if (lane == 0) {
+            atomicMin(&B.lmin, lmin);
+            atomicMax(&B.lmax, lmax);
+        }
+        uint32_t off = inc - loc;
+        for (int i = 0; i < w; ++i) off += B.wsum[i];
+        for (int j = j0; j < j1; ++j) {
+            pref[j] = off;
+            off += (uint32_t)max(0, (int)gL[lr0 + j] - k);
+        }
+        if (bt == NB - 1) pref[r] = off;   // the last builder covers the last read (or none)
+        builders_sync(NB);
+        if (bt == 0) E.ulen = (r > 0 && B.lmin == B.lmax) ? B.lmax : -2;   // -2: lengths differ
+    }
 }
 
 template <bool INL, bool GT>
@@ -608,8 +666,12 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
     const volatile int *stop = &B.overflow;
     const int k = T.k, KW = T.KW;
     constexpr int NW = INL ? 2 : MAX_KW;   // inline keys: k <= 63 fits two words
-    constexpr int BATCH = GT ? 4 : 2;      // positions in flight per thread (register budget)
-    if (GT && INL) {   // global-memory table: batched passes (positions in flight hide L2 latency)
+#ifndef LA_SMEM_BATCH
+#define LA_SMEM_BATCH 1
+#endif
+    constexpr int BATCH = GT ? 4 : (LA_SMEM_BATCH > 1 ? LA_SMEM_BATCH : 2);   // positions in flight per thread
+    constexpr bool BATCHED = GT || LA_SMEM_BATCH > 1;   // measured: batching helps the L2 tables only
+    if (INL && BATCHED) {   // batched passes (independent positions in flight hide L2 latency)
         if (mbits) {
             for_each_vote4<NW, BATCH>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
                            [&](const KmerN<NW> (&Kq)[BATCH], uint32_t, int, const uint32_t (&)[BATCH], uint32_t, uint32_t vm) {
@@ -660,7 +722,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
     // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
     if (mbits) {
         for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const KmerN<NW> &K, uint32_t, int, uint32_t, bool) {
+                      [&](const KmerN<NW> K, uint32_t, int, uint32_t, bool) {
                           const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
                           const uint32_t bit = 1u << (fi & 31);
                           if (!(B2[fi >> 5] & bit)) {
@@ -674,7 +736,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
     // ---- build (Alg 1) ----
     const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
     for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const KmerN<NW> &K, uint32_t rid, int p, uint32_t nb, bool hi) {
+                      [&](const KmerN<NW> K, uint32_t rid, int p, uint32_t nb, bool hi) {
                           const uint64_t h = hash_kmer(K, KW);
                           if (mbits) {
                               const uint32_t fi = filt_index(h, mbits);
@@ -931,17 +993,21 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         const int ulen = E.ulen;
         // shared-memory tables: stage the end's reads (coalesced 16 B copies); the XL class streams
         // them from HBM/L2 instead
-        const uint64_t *gR = rseq, *gQ = rqc;
-        const uint16_t *gL = rlen;
-        const uint8_t *gF = rflag;
-        long long lr0 = r0;   // first read index in (gR, gQ, gL, gF)
+        // shared-memory tables: the end's reads are staged in shared memory (coalesced 16 B copies) and
+        // every builder access is a plain LDS (the pointers below are shared-memory pointers whenever
+        // !GT, so the compiler emits LDS, not generic loads); the XL class streams them from HBM/L2.
         unsigned char *stage = tbase + FX.off_tab;
         const bool no_room = !GT && stage_bytes(r, SW) + pref_bytes(r) + 64u * 24u > FX.tab_bytes;
+        uint64_t *sR = (uint64_t *)stage;
+        uint64_t *sQ = sR + (size_t)r * SW;
+        uint16_t *sL = (uint16_t *)(sQ + (size_t)r * SW);
+        uint8_t *sF = (uint8_t *)(sL + r);
+        const uint64_t *gR = GT ? rseq : sR;
+        const uint64_t *gQ = GT ? rqc : sQ;
+        const uint16_t *gL = GT ? rlen : sL;
+        const uint8_t *gF = GT ? rflag : sF;
+        const long long lr0 = GT ? r0 : 0;   // first read index in (gR, gQ, gL, gF)
         if (!GT && !no_room) {
-            uint64_t *sR = (uint64_t *)stage;
-            uint64_t *sQ = sR + (size_t)r * SW;
-            uint16_t *sL = (uint16_t *)(sQ + (size_t)r * SW);
-            uint8_t *sF = (uint8_t *)(sL + r);
             const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
             const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
             const int n4 = r * SW / 2;   // SW is even
@@ -953,60 +1019,13 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                 sL[i] = __ldg(&rlen[r0 + i]);
                 sF[i] = __ldg(&rflag[r0 + i]);
             }
-            gR = sR;
-            gQ = sQ;
-            gL = sL;
-            gF = sF;
-            lr0 = 0;
             builders_sync(NB);
         }
         // positions with a following base, per read (exclusive prefix, pref[r] = U) -> table plan
         uint32_t *pref = (uint32_t *)(stage + (GT ? 0u : stage_bytes(r, SW)));
         if (no_room) {   // the reads alone do not fit this CTA's shared memory: no table (overflow)
-        } else if (ulen >= 0) {   // all reads of the end have length ulen: arithmetic, no loads
-            const uint32_t np = (uint32_t)max(0, ulen - k);
-            for (int j = bt; j <= r; j += NB) pref[j] = (uint32_t)j * np;
-            builders_sync(NB);
         } else {
-            const int per = (r + NB - 1) / NB;
-            const int j0 = min(r, bt * per), j1 = min(r, j0 + per);
-            uint32_t loc = 0;
-            int lmin = 1 << 30, lmax = -1;
-            for (int j = j0; j < j1; ++j) {
-                const int l = gL[lr0 + j];
-                loc += (uint32_t)max(0, l - k);
-                lmin = min(lmin, l);
-                lmax = max(lmax, l);
-            }
-            const int lane = bt & 31, w = bt >> 5;
-            uint32_t inc = loc;
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t v = __shfl_up_sync(0xffffffffu, inc, o);
-                if (lane >= o) inc += v;
-            }
-            for (int o = 16; o; o >>= 1) {
-                lmin = min(lmin, __shfl_xor_sync(0xffffffffu, lmin, o));
-                lmax = max(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
-            }
-            if (bt == 0) {
-                B.lmin = 1 << 30;
-                B.lmax = -1;
-            }
-            if (lane == 31) B.wsum[w] = inc;
-            builders_sync(NB);
-            if (lane == 0) {
-                atomicMin(&B.lmin, lmin);
-                atomicMax(&B.lmax, lmax);
-            }
-            uint32_t off = inc - loc;
-            for (int i = 0; i < w; ++i) off += B.wsum[i];
-            for (int j = j0; j < j1; ++j) {
-                pref[j] = off;
-                off += (uint32_t)max(0, (int)gL[lr0 + j] - k);
-            }
-            if (bt == NB - 1) pref[r] = off;   // the last builder covers the last read (or none)
-            builders_sync(NB);
-            if (bt == 0) E.ulen = (r > 0 && B.lmin == B.lmax) ? B.lmax : -2;   // -2: lengths differ
+            read_prefix(B, E, pref, gL, lr0, r, k, ulen, bt, NB);
         }
         const uint32_t U = no_room ? 0u : pref[r];
         const long long tc = clock64();
@@ -1087,4 +1106,215 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     }
 }
 
+#ifndef LA_SMALL_MINB
+#define LA_SMALL_MINB(B) (768 / (B) > 0 ? 768 / (B) : 1)
+#endif
+// ---- k_small: one end per CTA, every thread builds, thread 0 walks -------------------------------
+// For the small-table classes the walk (a few thousand cycles) is short next to the build, so a
+// dedicated walker warp only halves the warps that build (ncu: the builders are latency-bound at
+// ~2 warps/SMSP).  Here all BLOCK threads build; after the link pass thread 0 walks while the others
+// wait at the barrier (other CTAs on the SM keep the issue slots busy).  The reads are staged in
+// shared memory once per end (not per attempt).
+template <int BLOCK>
+__global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
+    const int32_t *__restrict__ list, int n_list, int *__restrict__ work_ctr,
+    const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+    const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
+    const int64_t *__restrict__ eoff, const uint64_t *__restrict__ tail,
+    const uint64_t *__restrict__ tailN, const int32_t *__restrict__ clen, int SW, DevParams P,
+    uint32_t smem_bytes, uint8_t *__restrict__ walk_buf, int32_t *__restrict__ out_len,
+    uint8_t *__restrict__ out_term, uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
+    int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
+    unsigned char *__restrict__ gscratch, uint32_t gstride, unsigned long long *__restrict__ prof) {
+    (void)gscratch;
+    (void)gstride;
+    constexpr int NB = BLOCK;
+    extern __shared__ __align__(16) unsigned char sm[];
+    __shared__ EndSlot E;
+    __shared__ BuildCtl B;
+    __shared__ int s_done;
+    const int bt = threadIdx.x;
+    const SmemFixed FX = smem_fixed(P.W, smem_bytes, 0u, true);
+    const int Wp = (P.W + 15) & ~15;
+    uint8_t *wstr = sm + FX.off_walk;   // two walk strings: current / best
+    uint32_t *info = (uint32_t *)sm;
+    unsigned long long acc_ins = 0, acc_steps = 0, acc_att = 0, n_filtered = 0;
+    long long b_t[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // leader cycles: fetch, prefix, clear, filter, build, link, -, walk
+    for (;;) {
+        const long long ta = clock64();
+        if (bt == 0) {
+            const int idx = atomicAdd(work_ctr, 1);
+            B.skip = idx >= n_list;
+            if (!B.skip) {
+                const int e = list[idx];
+                E.e = e;
+                E.r0 = eoff[e];
+                E.r = (int)(eoff[e + 1] - E.r0);
+                E.ulen = -1;
+                E.kmax_eff = min(P.k_max, (int)clen[e]);
+                E.k = P.k_start;
+                E.shift = 0;
+                E.attempts = 0;
+                E.best_len = -1;
+                E.best_term = T_DEADEND;
+                E.best_k = 0;
+                E.best_buf = 1;
+                E.ins = 0;
+                E.steps = 0;
+            }
+        }
+        __syncthreads();
+        if (B.skip) break;
+        const int e = E.e;
+        const int r = E.r;
+        const long long r0 = E.r0;
+        // stage the end's reads once (coalesced 16 B copies)
+        unsigned char *stage = sm + FX.off_tab;
+        bool ovf = stage_bytes(r, SW) + pref_bytes(r) + 64u * 24u > FX.tab_bytes;
+        uint64_t *sR = (uint64_t *)stage;
+        uint64_t *sQ = sR + (size_t)r * SW;
+        uint16_t *sL = (uint16_t *)(sQ + (size_t)r * SW);
+        uint8_t *sF = (uint8_t *)(sL + r);
+        if (!ovf) {
+            const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
+            const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
+            const int n4 = r * SW / 2;   // SW is even
+            for (int i = bt; i < n4; i += NB) {
+                ((uint4 *)sR)[i] = __ldg(&a4[i]);
+                ((uint4 *)sQ)[i] = __ldg(&b4[i]);
+            }
+            for (int i = bt; i < r; i += NB) {
+                sL[i] = __ldg(&rlen[r0 + i]);
+                sF[i] = __ldg(&rflag[r0 + i]);
+            }
+        }
+        uint32_t *pref = (uint32_t *)(stage + stage_bytes(r, SW));
+        const int Tn = min((int)clen[e], 128);
+        const uint64_t *tail_e = tail + (size_t)e * TAIL_W;
+        const uint64_t n0 = tailN[2 * (size_t)e], n1 = tailN[2 * (size_t)e + 1];
+        __syncthreads();
+        b_t[0] += clock64() - ta;
+        while (!ovf) {   // attempts (k schedule)
+            const long long tb = clock64();
+            const int k = E.k;
+            const int KW = kwords(k);
+            read_prefix(B, E, pref, sL, 0, r, k, E.ulen, bt, NB);
+            const uint32_t U = pref[r];
+            SmemTab TB = smem_tab(FX, U, P.V >= 2, key_bytes(k), r, false, SW);
+            if (TB.cap < min_table_cap(BLOCK)) {
+                ovf = true;
+                break;
+            }
+            const uint32_t mbits = TB.mwords * 32u;
+            if (mbits) ++n_filtered;
+            uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);
+            uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
+            TabCtx T;
+            T.keys = (uint64_t *)(sm + TB.off_keys);
+            T.c32 = (uint32_t *)(sm + TB.off_cnts);
+            T.cap = TB.cap;
+            T.rseq = sR;
+            T.SW = SW;
+            T.k = k;
+            T.KW = KW;
+            if (bt == 0) {
+                B.overflow = 0;
+                B.nclaim = 0;
+            }
+            const long long tc = clock64();
+            {
+                const uint4 z = make_uint4(0, 0, 0, 0);
+                uint4 *a = (uint4 *)T.keys;
+                const uint32_t n16 = (TB.cap * (key_bytes(k) + cnt_bytes(false))) / 16u;
+                for (uint32_t i = bt; i < n16; i += NB) a[i] = z;
+                for (uint32_t i = bt; i < 2u * TB.mwords; i += NB) B1[i] = 0;
+            }
+            __syncthreads();
+            const long long td = clock64();
+            long long t_filter = td, t_build = td;
+            if (inline_keys(k))
+                build_link<true, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
+                                        NB, t_filter, t_build);
+            else
+                build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
+                                         NB, t_filter, t_build);
+            __syncthreads();
+            const long long te = clock64();
+            b_t[1] += tc - tb;
+            b_t[2] += td - tc;
+            b_t[3] += t_filter - td;
+            b_t[4] += t_build - t_filter;
+            b_t[5] += te - t_build;
+            if (B.overflow) {
+                ovf = true;
+                break;
+            }
+            if (bt == 0) {
+                // ---- walk (Alg 2) over the successor links ----
+                E.ins += U;
+                uint8_t *wb = wstr + (E.best_buf ^ 1) * Wp;
+                uint32_t node = B.start == NONE ? NEXT_NONE : B.start;
+                int len = 0, term = T_MAXLEN;
+                unsigned long long steps = 0;
+                for (int i = 0; i < P.W; ++i) {
+                    ++steps;   // a lookup; the loop check of a present k-mer precedes it (below)
+                    if (node == NEXT_NONE) { term = T_DEADEND; break; }
+                    const uint32_t inf = info[node];
+                    if (inf & 8u) { term = T_LOOP; --steps; break; }   // visited: loop check before lookup
+                    info[node] = inf | 8u;
+                    const uint32_t code = inf & 7u;
+                    if (code == CODE_FORK) { term = T_FORK; break; }
+                    if (code == CODE_DEADEND) { term = T_DEADEND; break; }
+                    wb[len++] = "ACGT"[code];
+                    node = inf >> 4;
+                }
+                E.attempts += 1;
+                E.steps += steps;
+                if (len > E.best_len) {   // longest walk, earliest on ties (reading #11)
+                    E.best_len = len;
+                    E.best_term = term;
+                    E.best_k = E.k;
+                    E.best_buf ^= 1;
+                }
+                int kk = E.k, sh = E.shift;
+                s_done = next_k(term, kk, sh, E.kmax_eff, P) ? 1 : 0;
+                E.k = kk;
+                E.shift = sh;
+            }
+            __syncthreads();
+            b_t[7] += clock64() - te;
+            if (s_done) break;
+        }
+        if (ovf) {   // table or counter overflow: the global path redoes this end from scratch
+            if (bt == 0) ovf_list[atomicAdd(n_ovf, 1)] = e;
+        } else {
+            const int bl = E.best_len;
+            const uint8_t *bw = wstr + E.best_buf * Wp;
+            uint8_t *dst = walk_buf + (size_t)e * P.W;
+            for (int i = bt; i < bl; i += NB) dst[i] = bw[i];
+            if (bt == 0) {
+                out_len[e] = bl;
+                out_term[e] = (uint8_t)E.best_term;
+                out_k[e] = (uint8_t)E.best_k;
+                out_att[e] = (uint8_t)E.attempts;
+                acc_ins += E.ins;
+                acc_steps += E.steps;
+                acc_att += E.attempts;
+            }
+        }
+        __syncthreads();   // E and the staged reads are reused by the next end
+    }
+    if (bt == 0) {
+        atomicAdd(&gstats->inserts, acc_ins);
+        atomicAdd(&gstats->steps, acc_steps);
+        atomicAdd(&gstats->attempts, acc_att);
+        atomicAdd(&gstats->filtered, n_filtered);
+        if (prof) {
+            for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
+            atomicAdd(&prof[7], (unsigned long long)b_t[7]);
+        }
+    }
+}
+
 }  // namespace la
+

@@ -64,6 +64,7 @@ struct la_ctx {
     int cls_threads[N_SMEM_CLASSES] = {64, 128, 256, 256, 512};
     int cls_ctas[N_SMEM_CLASSES] = {12, 6, 3, 2, 1};   // resident CTAs per SM of each shared-memory class
     uint32_t cls_bytes[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};   // dynamic shared memory per CTA
+    uint32_t small_mask = 0x3u;   // classes run by k_small (one end per CTA, no walker warp)
     la_params params{};
     DevParams dp{};
     Encoded enc, spare;   // current encoding; la_load_batch fills `spare` and swaps on success
@@ -190,6 +191,7 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
             ++q;
         }
     }
+    if (const char *m = getenv("LA_SMALL_MASK")) ctx->small_mask = (uint32_t)strtoul(m, nullptr, 0);
     // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
     for (int i = 0; i < N_SMEM_CLASSES; ++i) {
         size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - 512 /* static */;
@@ -217,6 +219,12 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         attr_ok &= cudaFuncSetAttribute(k_smem<192, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<96>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<192>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_small<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
     }
     if (!attr_ok) {
         cudaGetLastError();
@@ -554,6 +562,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
             pb.b[i] = force_global ? 0u : ctx->cls_bytes[i];
             pb.t[i] = (uint32_t)ctx->cls_threads[i];
         }
+        pb.single = ctx->small_mask;
         if (force_smem) pb.b[0] = 0xffffffffu;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
             P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
@@ -631,15 +640,35 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
                                       P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                         \
                                       P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,                          \
                                       (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr)
-            switch (ctx->cls_threads[c]) {
-                case 64: LA_LAUNCH_SMEM(64); break;
-                case 96: LA_LAUNCH_SMEM(96); break;
-                case 192: LA_LAUNCH_SMEM(192); break;
-                case 128: LA_LAUNCH_SMEM(128); break;
-                case 256: LA_LAUNCH_SMEM(256); break;
-                default: LA_LAUNCH_SMEM(512); break;
+#define LA_LAUNCH_SMALL(B)                                                                                  \
+    k_small<B><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen),  \
+                                       P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail),            \
+                                       P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                \
+                                       P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                      \
+                                       P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                        \
+                                       P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,                         \
+                                       (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr)
+            if ((ctx->small_mask >> c) & 1u) {
+                switch (ctx->cls_threads[c]) {
+                    case 64: LA_LAUNCH_SMALL(64); break;
+                    case 96: LA_LAUNCH_SMALL(96); break;
+                    case 192: LA_LAUNCH_SMALL(192); break;
+                    case 128: LA_LAUNCH_SMALL(128); break;
+                    case 256: LA_LAUNCH_SMALL(256); break;
+                    default: LA_LAUNCH_SMALL(512); break;
+                }
+            } else {
+                switch (ctx->cls_threads[c]) {
+                    case 64: LA_LAUNCH_SMEM(64); break;
+                    case 96: LA_LAUNCH_SMEM(96); break;
+                    case 192: LA_LAUNCH_SMEM(192); break;
+                    case 128: LA_LAUNCH_SMEM(128); break;
+                    case 256: LA_LAUNCH_SMEM(256); break;
+                    default: LA_LAUNCH_SMEM(512); break;
+                }
             }
 #undef LA_LAUNCH_SMEM
+#undef LA_LAUNCH_SMALL
             CKL();
         }
         if (c == 2) CK(cudaEventRecord(ctx->ev[5], st));   // after the 1- and 2-CTA/SM classes
