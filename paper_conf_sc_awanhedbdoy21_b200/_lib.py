@@ -9,7 +9,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO = os.path.join(HERE, "liblocassm.so")
+SO = os.environ.get("LA_SO") or os.path.join(HERE, "liblocassm.so")   # LA_SO: debug builds (tools/)
 
 LA_OK, LA_ERR_INVALID_ARG, LA_ERR_OOM, LA_ERR_CUDA, LA_ERR_STATE, LA_ERR_CAPACITY = 0, -1, -2, -3, -4, -5
 LA_MEM_HOST, LA_MEM_DEVICE = 0, 1

@@ -298,6 +298,36 @@ struct TabCtx {   // what a table operation needs
     int SW, k, KW;
 };
 
+// One vote for base b of slot s: a single atomic per vote.  Counter words hold the
+// high-tier votes (q >= q_hi) and the low-only votes (q_lo <= q < q_hi) separately; the low tier of
+// reading #1 is their sum (votes_of).  Shared memory: 8-bit fields of two u32 words (lo-only, hi),
+// a field about to carry flags the end for the global path; global (XL): 8 x u32, RED.ADD.
+template <bool GT>
+__device__ __forceinline__ void vote_add(const TabCtx &T, uint32_t s, uint32_t b, bool hi, volatile int *ovf) {
+    if (GT) {
+        atomicAdd(&T.c32[8 * (size_t)s + (hi ? 4u : 0u) + b], 1u);
+    } else {
+        const uint32_t old = atomicAdd(&T.c32[2 * s + (hi ? 1u : 0u)], 1u << (8 * b));
+        if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit counter would carry
+    }
+}
+
+template <bool GT>
+__device__ __forceinline__ void votes_of(const TabCtx &T, uint32_t s, uint32_t lo[4], uint32_t hi[4]) {
+    if (GT) {
+        const uint4 a = ((const uint4 *)T.c32)[2 * (size_t)s], c = ((const uint4 *)T.c32)[2 * (size_t)s + 1];
+        hi[0] = c.x; hi[1] = c.y; hi[2] = c.z; hi[3] = c.w;
+        lo[0] = a.x + c.x; lo[1] = a.y + c.y; lo[2] = a.z + c.z; lo[3] = a.w + c.w;
+    } else {
+        const uint2 w = ((const uint2 *)T.c32)[s];
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+            hi[b] = (w.y >> (8 * b)) & 0xffu;
+            lo[b] = ((w.x >> (8 * b)) & 0xffu) + hi[b];
+        }
+    }
+}
+
 template <bool INL, int NW>
 __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> &K, uint64_t h) {
     uint32_t s = slot_of(h, T.cap);
@@ -374,14 +404,7 @@ __device__ __forceinline__ void tab_insert(const TabCtx &T, const KmerN<NW> &K, 
             s = (s + 1 == T.cap) ? 0 : s + 1;
         }
     }
-    if (GT) {   // 8 x u32 in L2: RED.ADD, nothing to wait for
-        atomicAdd(&T.c32[8 * (size_t)s + b], 1u);
-        if (hi) atomicAdd(&T.c32[8 * (size_t)s + 4 + b], 1u);
-    } else {    // 32-bit ATOMS.ADD (a 64-bit shared-memory add compiles to a CAS loop)
-        const uint32_t old = atomicAdd(&T.c32[2 * s], 1u << (8 * b));
-        if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit lo counter would carry
-        if (hi) atomicAdd(&T.c32[2 * s + 1], 1u << (8 * b));  // hi <= lo: cannot carry first
-    }
+    vote_add<GT>(T, s, b, hi, ovf);
 }
 
 // Every voting occurrence of the end's reads (staged in shared memory, or streamed from global memory
@@ -442,119 +465,249 @@ __device__ __forceinline__ void for_each_vote(const uint64_t *__restrict__ rseq,
     }
 }
 
-// Batched variant for global-memory (XL) tables: positions are processed four at a time so that the
-// four hashes, filter probes and table probes are independent L2 requests in flight together.
-// f4(Kq, rid, p0, nbq, himask, vmask): bit u of vmask = position p0+u votes; of himask = high tier.
-template <int NW, int BATCH, typename F4>
-__device__ __forceinline__ void for_each_vote4(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
-                                               const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
-                                               const uint32_t *pref, int64_t r0, int r, int SW, int k, int KW,
-                                               int bt, int NB, const volatile int *stop, F4 &&f4) {
-    const uint32_t total = pref[r];
-    uint32_t cur = (uint32_t)(((uint64_t)total * (uint32_t)bt) / (uint32_t)NB);
-    const uint32_t end = (uint32_t)(((uint64_t)total * (uint32_t)(bt + 1)) / (uint32_t)NB);
-    if (cur >= end) return;
-    int lo = 0, hi = r;
-    while (hi - lo > 1) {
-        const int mid = (lo + hi) >> 1;
-        if (pref[mid] <= cur) lo = mid; else hi = mid;
+#ifdef LA_PROBE_STATS
+// debug build only: [0] warp_insert calls, [1] probe rounds, [2] inserting lanes, [3] claims,
+// [4] lookup calls, [5] lookup rounds, [6] looking-up lanes, [7] sum of table loads at link (claims*1000/cap)
+__device__ unsigned long long g_probe_stats[8];
+#define LA_PSTAT(i, v) atomicAdd(&g_probe_stats[i], (unsigned long long)(v))
+#else
+#define LA_PSTAT(i, v) ((void)0)
+#endif
+
+// ---- warp-convergent passes (k <= 63, inline keys) --------------------------------------------
+// Lane-per-position: builder warp w owns the contiguous range [w*U/NW, (w+1)*U/NW) of the end's
+// numbered positions (pref, read by read) and its 32 lanes take 32 consecutive positions per
+// iteration, so every lane runs the same iteration count and the hash / probe / vote code executes
+// with the whole warp active (the per-thread rolling loops ran at ~5 of 32 lanes, ncu r01).  Each lane
+// extracts its k-mer from the packed read (3 words, funnel shifts) — no rolling, no read-boundary
+// branches; consecutive lanes read the same or adjacent words (broadcast).
+struct PosV {            // one lane's position
+    KmerN<2> K;
+    uint32_t nb;         // following base (Alg 1 line 6)
+    bool vote, hi;       // votes at all (q >= q_lo and no N in the window) / in the high tier
+};
+
+__device__ __forceinline__ uint64_t nmask_word(uint64_t q) { return q & (q >> 1) & 0x5555555555555555ull; }
+
+// position p of read row (R, Q); has_n: the read contains an N (rflag)
+__device__ __forceinline__ PosV pos_value(const uint64_t *R, const uint64_t *Q, int p, int k, int KW, int SW,
+                                          bool has_n) {
+    PosV v;
+    const int q = p >> 5, s = (p & 31) << 1;
+    const int q2 = min(q + 2, SW - 1);   // word q+2 is only needed when the window reaches it
+    const uint64_t r0 = R[q], r1 = R[q + 1], r2 = R[q2];
+    const int b1 = 2 * k - 64;           // bits of word 1 (<= 0: k <= 32)
+    const uint64_t m0 = b1 >= 0 ? ~0ull : (~0ull << (64 - 2 * k));
+    const uint64_t m1 = b1 > 0 ? (~0ull << (64 - b1)) : 0ull;
+    v.K.w[0] = funnel64(r0, r1, s) & m0;
+    v.K.w[1] = funnel64(r1, r2, s) & m1;
+    (void)KW;
+    const int i = p + k, wi = i >> 5, d = wi - q;   // following base, word q+d (d in 0..2)
+    const uint64_t rw = d == 0 ? r0 : (d == 1 ? r1 : r2);
+    const int sh = 62 - ((i & 31) << 1);
+    v.nb = (uint32_t)(rw >> sh) & 3u;
+    const uint32_t nq = (uint32_t)(Q[wi] >> sh) & 3u;
+    v.vote = nq - 1u < 2u;
+    v.hi = nq == 2u;
+    if (has_n) {   // reading #5: a k-mer with an N has no entry (rare: ~1% of reads)
+        const uint64_t n0 = nmask_word(Q[q]), n1 = nmask_word(Q[q + 1]), n2 = nmask_word(Q[q2]);
+        if ((funnel64(n0, n1, s) & m0) | (funnel64(n1, n2, s) & m1)) v.vote = false;
     }
-    int j = lo;
-    while (pref[j + 1] <= cur) ++j;
-    int p = (int)(cur - pref[j]);
-    while (cur < end) {
-        if (*stop) return;
-        const int64_t rid = r0 + j;
-        const int npos = (int)(pref[j + 1] - pref[j]);
-        const int pe = min(npos, p + (int)(end - cur));
-        const uint64_t *R = rseq + rid * SW;
-        const uint64_t *Q = rqc + rid * SW;
-        KmerN<NW> K = extract_kmer<NW>(R, p, k, KW);
-        int lastN = -1;
-        if (rflag[rid])
-            for (int i = p; i < p + k; ++i)
-                if (get2(Q, i) == 3u) lastN = i;
-        int wi = (p + k) >> 5;
-        uint64_t wR = R[wi], wQ = Q[wi];
-        for (int q = p; q < pe; q += BATCH) {
-            KmerN<NW> Kq[BATCH];
-            uint32_t nbq[BATCH];
-            uint32_t vm = 0, hm = 0;
-#pragma unroll
-            for (int u = 0; u < BATCH; ++u) {
-                Kq[u] = K;
-                nbq[u] = 0;
-                const int qq = q + u;
-                if (qq < pe) {
-                    const int i = qq + k;
-                    if ((i >> 5) != wi) {
-                        wi = i >> 5;
-                        wR = R[wi];
-                        wQ = Q[wi];
-                    }
-                    const int sh = 62 - ((i & 31) << 1);
-                    const uint32_t nb = (uint32_t)(wR >> sh) & 3u;
-                    const uint32_t nq = (uint32_t)(wQ >> sh) & 3u;
-                    if (nq - 1u < 2u && lastN < qq) {
-                        vm |= 1u << u;
-                        if (nq == 2u) hm |= 1u << u;
-                    }
-                    if (nq == 3u) lastN = i;
-                    nbq[u] = nb;
-                    roll_kmer(K, k, KW, nb);
-                }
-            }
-            if (vm) f4(Kq, (uint32_t)rid, q, nbq, hm, vm);
+    return v;
+}
+
+// f(act, v): act = this lane has a position this iteration (warp-uniform call).
+template <typename F>
+__device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+                                               const uint8_t *__restrict__ rflag, const uint32_t *pref,
+                                               long long r0, int r, int SW, int k, int KW, int wid, int nwarps,
+                                               int lane, const volatile int *stop, F &&f) {
+    const uint32_t total = pref[r];
+    const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
+    const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
+    if (wb >= we) return;
+    uint32_t g = wb + lane;
+    int j;
+    {   // read j with pref[j] <= g < pref[j+1]
+        const uint32_t gg = min(g, we - 1);
+        int lo = 0, hi = r;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (pref[mid] <= gg) lo = mid; else hi = mid;
         }
-        cur += (uint32_t)(pe - p);
-        ++j;
-        p = 0;
-        while (cur < end && pref[j + 1] == pref[j]) ++j;
+        j = lo;
+    }
+    for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
+        if (__shfl_sync(0xffffffffu, *stop, 0)) return;
+        const bool act = g < we;
+        PosV v;
+        v.vote = false;
+        if (act) {
+            uint32_t pj = pref[j + 1];
+            while (pj <= g) pj = pref[++j + 1];   // crossed into a later read (skips reads without positions)
+            const long long rid = r0 + j;
+            v = pos_value(rseq + rid * SW, rqc + rid * SW, (int)(g - pref[j]), k, KW, SW, rflag[rid] != 0);
+        }
+        f(act && v.vote, v);
     }
 }
 
-// Four inline-key inserts with interleaved probing: each round issues the probe loads of all pending
-// inserts before resolving any of them (s[u]: start slot of insert u).
-template <bool GT, int NW, int BATCH>
-__device__ __forceinline__ void tab_insert4_inline(const TabCtx &T, const KmerN<NW> (&Kq)[BATCH], uint32_t (&s)[BATCH],
-                                                   const uint32_t (&nbq)[BATCH], uint32_t hm, uint32_t pm, int *nclaim,
-                                                   int claim_limit, volatile int *ovf) {
-    while (pm) {
-        uint64_t x[BATCH], y[BATCH];
+// Lane-per-run variant: warp iteration = 32*RUN consecutive positions, lane l takes the RUN positions
+// base + l*RUN + i.  The k-mer is extracted once per run (or when the run crosses into the next read)
+// and rolled (next_kmer, Alg 2 line 15) for the others, so a position costs a roll, not an extraction.
+// f(act, v) is called RUN times per iteration by the whole warp.
+template <int RUN, typename F>
+__device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+                                          const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
+                                          int r, int SW, int k, int KW, int wid, int nwarps, int lane,
+                                          const volatile int *stop, F &&f) {
+    const uint32_t total = pref[r];
+    const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
+    const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
+    if (wb >= we) return;
+    constexpr uint32_t SPAN = 32u * RUN;
+    uint32_t g = wb + (uint32_t)lane * RUN;
+    int j;
+    {   // read j with pref[j] <= g < pref[j+1]
+        const uint32_t gg = min(g, we - 1);
+        int lo = 0, hi = r;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (pref[mid] <= gg) lo = mid; else hi = mid;
+        }
+        j = lo;
+    }
+    for (uint32_t base = wb; base < we; base += SPAN, g += SPAN) {
+        if (__shfl_sync(0xffffffffu, *stop, 0)) return;
+        KmerN<2> K;
+        K.w[0] = K.w[1] = 0;
+        int p = 0, lastN = -1, npos = 0;
+        const uint64_t *R = rseq, *Q = rqc;
+        bool flag = false;
+        // (re)start: extract the k-mer at position g (read j) — at the run start and at a read change
+        auto start = [&](uint32_t gpos) {
+            uint32_t pj = pref[j + 1];
+            while (pj <= gpos) pj = pref[++j + 1];   // skips reads without positions
+            const uint32_t pj0 = pref[j];
+            p = (int)(gpos - pj0);
+            npos = (int)(pj - pj0);
+            const long long rid = r0 + j;
+            R = rseq + rid * SW;
+            Q = rqc + rid * SW;
+            flag = rflag[rid] != 0;
+            K = extract_kmer<2>(R, p, k, KW);
+            lastN = -1;
+            if (flag)
+                for (int i = p; i < p + k; ++i)
+                    if (get2(Q, i) == 3u) lastN = i;
+        };
+        if (g < we) start(g);
 #pragma unroll
-        for (int u = 0; u < BATCH; ++u)
-            if ((pm >> u) & 1u) ld128v<GT>(&T.keys[2 * (size_t)s[u]], x[u], y[u]);
-#pragma unroll
-        for (int u = 0; u < BATCH; ++u) {
-            if (!((pm >> u) & 1u)) continue;
-            uint64_t a, bb;
-            inline_form(Kq[u], T.KW, a, bb);
-            bool found = false;
-            if (y[u] == 0) {
-                if (*ovf) { pm &= ~(1u << u); continue; }
-                cas128<GT>((void *)&T.keys[2 * (size_t)s[u]], 0ull, 0ull, a, bb, x[u], y[u]);
-                if (y[u] == 0) {
-                    found = true;
-                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
-                }
-            } else if (y[u] == bb && x[u] != a) {
-                x[u] = *(volatile uint64_t *)&T.keys[2 * (size_t)s[u]];
+        for (int i = 0; i < RUN; ++i) {
+            const uint32_t gi = g + (uint32_t)i;
+            const bool act = gi < we;
+            if (act && i > 0 && p >= npos) start(gi);   // the run crossed into the next read
+            PosV v;
+            v.vote = false;
+            v.nb = 0;
+            v.hi = false;
+            if (act) {
+                const int ii = p + k, sh = 62 - ((ii & 31) << 1);
+                v.nb = (uint32_t)(R[ii >> 5] >> sh) & 3u;
+                const uint32_t nq = (uint32_t)(Q[ii >> 5] >> sh) & 3u;
+                v.vote = nq - 1u < 2u && lastN < p;
+                v.hi = nq == 2u;
+                if (nq == 3u) lastN = ii;
             }
-            if (found || (x[u] == a && y[u] == bb)) {
-                if (GT) {
-                    atomicAdd(&T.c32[8 * (size_t)s[u] + nbq[u]], 1u);
-                    if ((hm >> u) & 1u) atomicAdd(&T.c32[8 * (size_t)s[u] + 4 + nbq[u]], 1u);
-                } else {
-                    const uint32_t old = atomicAdd(&T.c32[2 * s[u]], 1u << (8 * nbq[u]));
-                    if (((old >> (8 * nbq[u])) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit counter would carry
-                    if ((hm >> u) & 1u) atomicAdd(&T.c32[2 * s[u] + 1], 1u << (8 * nbq[u]));
-                }
-                pm &= ~(1u << u);
-            } else {
-                s[u] = (s[u] + 1 == T.cap) ? 0 : s[u] + 1;
+            v.K = K;
+            f(act && v.vote, v);
+            if (i + 1 < RUN && act) {
+                roll_kmer(K, k, KW, v.nb);
+                ++p;
             }
         }
     }
+}
+
+// Convergent insert of the lanes with `want` (Alg 1 line 5 + the vote): every probe round
+// is entered by the whole warp; claims are counted once per warp.
+template <bool GT>
+__device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const PosV &v, uint64_t h, int lane,
+                                            int *nclaim, int claim_limit, volatile int *ovf) {
+    uint32_t s = slot_of(h, T.cap);
+    const uint64_t a = v.K.w[0], bb = ~(T.KW >= 2 ? v.K.w[1] : 0ull);
+    bool pend = want, found = false;
+#ifdef LA_PROBE_STATS
+    { const unsigned m = __ballot_sync(0xffffffffu, want); if (lane == 0) { LA_PSTAT(0, 1); LA_PSTAT(2, __popc(m)); } }
+#endif
+    while (__any_sync(0xffffffffu, pend)) {
+        if (lane == 0) LA_PSTAT(1, 1);
+        bool claimed = false;
+        if (pend) {
+            uint64_t x, y;
+            ld128v<GT>(&T.keys[2 * (size_t)s], x, y);
+            if (y == 0) {   // looks empty: the CAS claims it or returns its true content
+                if (*ovf) {
+                    pend = false;
+                } else {
+                    cas128<GT>((void *)&T.keys[2 * (size_t)s], 0ull, 0ull, a, bb, x, y);
+                    if (y == 0) {
+                        claimed = true;
+                        x = a;
+                        y = bb;
+                    }
+                }
+            } else if (y == bb && x != a) {
+                // a 16 B load is not single-copy atomic: if it raced with the claiming CAS, word 0 may
+                // be stale — re-read it (a slot never changes once claimed)
+                x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
+            }
+            if (pend) {
+                if (x == a && y == bb) {
+                    pend = false;
+                    found = true;
+                } else {
+                    s = (s + 1 == T.cap) ? 0 : s + 1;
+                }
+            }
+        }
+        const unsigned cm = __ballot_sync(0xffffffffu, claimed);
+        if (cm && lane == __ffs(cm) - 1) {
+            const int n = __popc(cm);
+            LA_PSTAT(3, n);
+            if (atomicAdd(nclaim, n) + n > claim_limit) *ovf = 1;
+        }
+    }
+    if (found) vote_add<GT>(T, s, v.nb, v.hi, ovf);
+}
+
+// Convergent lookup (no insert): slot of K or NONE.
+template <bool GT>
+__device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, const KmerN<2> &K, uint64_t h) {
+    uint32_t s = slot_of(h, T.cap), res = NONE;
+    const uint64_t a = K.w[0], bb = ~(T.KW >= 2 ? K.w[1] : 0ull);
+    bool pend = want;
+    uint32_t n = 0;
+#ifdef LA_PROBE_STATS
+    { const unsigned m = __ballot_sync(0xffffffffu, want); if ((threadIdx.x & 31) == 0) { LA_PSTAT(4, 1); LA_PSTAT(6, __popc(m)); } }
+#endif
+    while (__any_sync(0xffffffffu, pend)) {
+        if ((threadIdx.x & 31) == 0) LA_PSTAT(5, 1);
+        if (pend) {
+            uint64_t x, y;
+            ld128v<GT>(&T.keys[2 * (size_t)s], x, y);
+            if (y == 0) {
+                pend = false;
+            } else if (x == a && y == bb) {
+                pend = false;
+                res = s;
+            } else {
+                s = (s + 1 == T.cap) ? 0 : s + 1;
+                if (++n >= T.cap) pend = false;
+            }
+        }
+    }
+    return res;
 }
 
 // ---- the kernel --------------------------------------------------------------------------------
@@ -656,6 +809,25 @@ __device__ __forceinline__ void read_prefix(BuildCtl &B, EndSlot &E, uint32_t *p
     }
 }
 
+// Slot-parallel pass after the build: ext(lo, hi) (reading #1, a5) and, for a base, the successor
+// k-mer's slot (next_kmer, Alg 2 line 15) -> info[s] = next << 4 | code.
+__device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
+    return (code < 4 ? (nxt == NONE ? NEXT_NONE : nxt) : NEXT_NONE) << 4 | (uint32_t)code;
+}
+
+#ifndef LA_RUN
+#define LA_RUN 1   // positions per lane per warp iteration: 1 = warp_positions (measured fastest), >1 = warp_runs
+#endif
+template <typename F>
+__device__ __forceinline__ void warp_pass(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+                                          const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
+                                          int r, int SW, int k, int KW, int wid, int nwarps, int lane,
+                                          const volatile int *stop, F &&f) {
+    if (LA_RUN > 1)
+        warp_runs<LA_RUN>(rseq, rqc, rflag, pref, r0, r, SW, k, KW, wid, nwarps, lane, stop, f);
+    else
+        warp_positions(rseq, rqc, rflag, pref, r0, r, SW, k, KW, wid, nwarps, lane, stop, f);
+}
 template <bool INL, bool GT>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
@@ -665,125 +837,138 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                            long long &t_filter, long long &t_build) {
     const volatile int *stop = &B.overflow;
     const int k = T.k, KW = T.KW;
-    constexpr int NW = INL ? 2 : MAX_KW;   // inline keys: k <= 63 fits two words
-#ifndef LA_SMEM_BATCH
-#define LA_SMEM_BATCH 1
-#endif
-    constexpr int BATCH = GT ? 4 : (LA_SMEM_BATCH > 1 ? LA_SMEM_BATCH : 2);   // positions in flight per thread
-    constexpr bool BATCHED = GT || LA_SMEM_BATCH > 1;   // measured: batching helps the L2 tables only
-    if (INL && BATCHED) {   // batched passes (independent positions in flight hide L2 latency)
+    const int lane = bt & 31, wid = bt >> 5, nwarps = NB >> 5;
+    const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
+    if (INL) {
+        // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
         if (mbits) {
-            for_each_vote4<NW, BATCH>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                           [&](const KmerN<NW> (&Kq)[BATCH], uint32_t, int, const uint32_t (&)[BATCH], uint32_t, uint32_t vm) {
-                               uint32_t fi[BATCH], w2[BATCH], need = 0;
-#pragma unroll
-                               for (int u = 0; u < BATCH; ++u)
-                                   if ((vm >> u) & 1u) {
-                                       fi[u] = filt_index(hash_kmer(Kq[u], KW), mbits);
-                                       w2[u] = *(volatile uint32_t *)&B2[fi[u] >> 5];
-                                   }
-                               uint32_t old[BATCH];
-#pragma unroll
-                               for (int u = 0; u < BATCH; ++u)
-                                   if (((vm >> u) & 1u) && !((w2[u] >> (fi[u] & 31)) & 1u)) {
-                                       old[u] = atomicOr(&B1[fi[u] >> 5], 1u << (fi[u] & 31));
-                                       need |= 1u << u;
-                                   }
-#pragma unroll
-                               for (int u = 0; u < BATCH; ++u)
-                                   if (((need >> u) & 1u) && ((old[u] >> (fi[u] & 31)) & 1u))
-                                       atomicOr(&B2[fi[u] >> 5], 1u << (fi[u] & 31));
+            warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                           [&](bool act, const PosV &v) {
+                               if (!act) return;
+                               const uint32_t fi = filt_index(hash_kmer(v.K, KW), mbits);
+                               const uint32_t bit = 1u << (fi & 31);
+                               if (!(*(volatile uint32_t *)&B2[fi >> 5] & bit)) {
+                                   const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                   if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                               }
                            });
             builders_sync(NB);
         }
         t_filter = clock64();
-        const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
-        for_each_vote4<NW, BATCH>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                       [&](const KmerN<NW> (&Kq)[BATCH], uint32_t, int, const uint32_t (&nbq)[BATCH], uint32_t hm, uint32_t vm) {
-                           uint32_t sl[BATCH], w2[BATCH], fi[BATCH];
-                           uint32_t pm = vm;
-#pragma unroll
-                           for (int u = 0; u < BATCH; ++u) {
-                               const uint64_t h = hash_kmer(Kq[u], KW);
-                               sl[u] = slot_of(h, T.cap);
-                               fi[u] = filt_index(h, mbits);
-                           }
+        // ---- build (Alg 1) ----
+        warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                       [&](bool act, const PosV &v) {
+                           const uint64_t h = hash_kmer(v.K, KW);
+                           bool want = act;
                            if (mbits) {
-#pragma unroll
-                               for (int u = 0; u < BATCH; ++u)
-                                   if ((vm >> u) & 1u) w2[u] = B2[fi[u] >> 5];
-#pragma unroll
-                               for (int u = 0; u < BATCH; ++u)
-                                   if (((vm >> u) & 1u) && !((w2[u] >> (fi[u] & 31)) & 1u)) pm &= ~(1u << u);
+                               const uint32_t fi = filt_index(h, mbits);
+                               want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
                            }
-                           if (pm) tab_insert4_inline<GT, NW, BATCH>(T, Kq, sl, nbq, hm, pm, &B.nclaim, claim_limit, &B.overflow);
+                           warp_insert<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
                        });
     } else {
-    // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
-    if (mbits) {
+        constexpr int NW = MAX_KW;
+        // ---- filter pass (REF keys, k >= 64: rare; per-thread rolling traversal) ----
+        if (mbits) {
+            for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
+                              [&](const KmerN<NW> K, uint32_t, int, uint32_t, bool) {
+                                  const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
+                                  const uint32_t bit = 1u << (fi & 31);
+                                  if (!(B2[fi >> 5] & bit)) {
+                                      const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                      if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                                  }
+                              });
+            builders_sync(NB);
+        }
+        t_filter = clock64();
         for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const KmerN<NW> K, uint32_t, int, uint32_t, bool) {
-                          const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
-                          const uint32_t bit = 1u << (fi & 31);
-                          if (!(B2[fi >> 5] & bit)) {
-                              const uint32_t old = atomicOr(&B1[fi >> 5], bit);
-                              if (old & bit) atomicOr(&B2[fi >> 5], bit);
-                          }
-                      });
-        builders_sync(NB);
-    }
-    t_filter = clock64();
-    // ---- build (Alg 1) ----
-    const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
-    for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                      [&](const KmerN<NW> K, uint32_t rid, int p, uint32_t nb, bool hi) {
-                          const uint64_t h = hash_kmer(K, KW);
-                          if (mbits) {
-                              const uint32_t fi = filt_index(h, mbits);
-                              if (!((B2[fi >> 5] >> (fi & 31)) & 1u)) return;
-                          }
-                          tab_insert<INL, GT, NW>(T, K, h, rid, p, nb, hi, &B.nclaim, claim_limit, &B.overflow);
-                      });
+                          [&](const KmerN<NW> K, uint32_t rid, int p, uint32_t nb, bool hi) {
+                              const uint64_t h = hash_kmer(K, KW);
+                              if (mbits) {
+                                  const uint32_t fi = filt_index(h, mbits);
+                                  if (!((B2[fi >> 5] >> (fi & 31)) & 1u)) return;
+                              }
+                              tab_insert<false, GT, NW>(T, K, h, rid, p, nb, hi, &B.nclaim, claim_limit, &B.overflow);
+                          });
     }
     builders_sync(NB);
     t_build = clock64();
     if (B.overflow) return;
+#ifdef LA_PROBE_STATS
+    if (bt == 0) LA_PSTAT(7, (unsigned long long)B.nclaim * 1000ull / T.cap);
+#endif
     // ---- ext rule + successor links (a5) into the end's info buffer ----
-    for (uint32_t s = bt; s < T.cap; s += NB) {
-        KmerN<NW> K;
-        if (INL) {
-            const ulonglong2 w = ((const ulonglong2 *)T.keys)[s];
-            if (w.y == 0) continue;
-#pragma unroll
-            for (int i = 0; i < NW; ++i) K.w[i] = 0;
-            K.w[0] = w.x;
-            if (NW > 1) K.w[NW > 1 ? 1 : 0] = KW >= 2 ? ~w.y : 0ull;
-        } else {
-            const uint64_t w = T.keys[s];
-            if (w == 0) continue;
-            K = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
-        }
-        uint32_t lo[4], hi[4];
-        if (GT) {
-            const uint4 a = ((const uint4 *)T.c32)[2 * (size_t)s], c = ((const uint4 *)T.c32)[2 * (size_t)s + 1];
-            lo[0] = a.x; lo[1] = a.y; lo[2] = a.z; lo[3] = a.w;
-            hi[0] = c.x; hi[1] = c.y; hi[2] = c.z; hi[3] = c.w;
-        } else {
-            const uint32_t lw = T.c32[2 * s], hw = T.c32[2 * s + 1];
-#pragma unroll
-            for (int b = 0; b < 4; ++b) {
-                lo[b] = (lw >> (8 * b)) & 0xffu;
-                hi[b] = (hw >> (8 * b)) & 0xffu;
+    if (INL) {
+        // Occupied slots (~30% of the table) are compacted into full warps first: each warp scans
+        // its chunks of 32 slots and queues the occupied ones in a one-slot-per-lane register queue;
+        // every full queue (and the final partial one) is linked with all lanes busy.
+        auto link_batch = [&](bool has, uint32_t s) {
+            KmerN<2> K;
+            K.w[0] = K.w[1] = 0;
+            int code = CODE_DEADEND;
+            if (has) {
+                const ulonglong2 w = ((const ulonglong2 *)T.keys)[s];
+                K.w[0] = w.x;
+                K.w[1] = KW >= 2 ? ~w.y : 0ull;
+                uint32_t lo[4], hi[4];
+                votes_of<GT>(T, s, lo, hi);
+                code = ext_rule(lo, hi, P.V, P.F);
+                if (code < 4) roll_kmer(K, k, KW, (uint32_t)code);
+            }
+            const uint32_t t = warp_lookup<GT>(T, has && code < 4, K, hash_kmer(K, KW));
+            if (has) info[s] = link_info(code, t);
+        };
+#ifndef LA_LINK_COMPACT
+#define LA_LINK_COMPACT 1
+#endif
+        if (!LA_LINK_COMPACT) {
+            for (uint32_t base = (uint32_t)wid * 32u; base < T.cap; base += (uint32_t)NB) {
+                const uint32_t s = base + lane;
+                link_batch(s < T.cap && ((const ulonglong2 *)T.keys)[min(s, T.cap - 1)].y != 0, s);
             }
         }
-        const int code = ext_rule(lo, hi, P.V, P.F);
-        uint32_t nxt = NEXT_NONE;
-        if (code < 4) {
-            roll_kmer(K, k, KW, (uint32_t)code);
-            const uint32_t t = tab_lookup<INL, NW>(T, K, hash_kmer(K, KW));
-            nxt = t == NONE ? NEXT_NONE : t;
+        uint32_t qs = 0;
+        int qn = 0;
+        for (uint32_t base = (uint32_t)wid * 32u; LA_LINK_COMPACT; base += (uint32_t)NB) {
+            const bool more = base < T.cap;   // warp-uniform
+            uint32_t m = 0;
+            if (more) {
+                const uint32_t s = base + lane;
+                bool occ = false;
+                if (s < T.cap) occ = ((const ulonglong2 *)T.keys)[s].y != 0;
+                m = __ballot_sync(0xffffffffu, occ);
+            }
+            const int n = __popc(m), tot = qn + n;
+            const int t = lane - qn;   // rank (in m) of the new slot this lane takes
+            const uint32_t mine = lane < qn ? qs : (t < n ? base + __fns(m, 0, t + 1) : 0u);
+            if (tot >= 32 || (!more && tot > 0)) {
+                link_batch(lane < tot, mine);
+                const int t2 = 32 - qn + lane;   // leftover ranks 32-qn .. n-1 -> lanes 0..
+                qn = tot > 32 ? tot - 32 : 0;
+                qs = lane < qn ? base + __fns(m, 0, t2 + 1) : 0u;
+            } else {
+                qs = mine;
+                qn = tot;
+            }
+            if (!more) break;
         }
-        info[s] = (nxt << 4) | (uint32_t)code;
+    } else {
+        constexpr int NW = MAX_KW;
+        for (uint32_t s = bt; s < T.cap; s += NB) {
+            const uint64_t w = T.keys[s];
+            if (w == 0) continue;
+            KmerN<NW> K = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
+            uint32_t lo[4], hi[4];
+            votes_of<GT>(T, s, lo, hi);
+            const int code = ext_rule(lo, hi, P.V, P.F);
+            uint32_t nxt = NONE;
+            if (code < 4) {
+                roll_kmer(K, k, KW, (uint32_t)code);
+                nxt = tab_lookup<false, NW>(T, K, hash_kmer(K, KW));
+            }
+            info[s] = link_info(code, nxt);
+        }
     }
     if (bt == 0) {
         // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
@@ -795,8 +980,13 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             uint64_t Tw[TAIL_W];
 #pragma unroll
             for (int i = 0; i < TAIL_W; ++i) Tw[i] = tail_e[i];
-            const KmerN<NW> K = extract_kmer<NW>(Tw, p, k, KW);
-            st = tab_lookup<INL, NW>(T, K, hash_kmer(K, KW));
+            if (INL) {
+                const KmerN<2> K = extract_kmer<2>(Tw, p, k, KW);
+                st = tab_lookup<true, 2>(T, K, hash_kmer(K, KW));
+            } else {
+                const KmerN<MAX_KW> K = extract_kmer<MAX_KW>(Tw, p, k, KW);
+                st = tab_lookup<false, MAX_KW>(T, K, hash_kmer(K, KW));
+            }
         }
         B.start = st;
     }

@@ -269,6 +269,16 @@ extern "C" la_status la_get_stats(const la_ctx *ctx, la_stats *out) {
 }
 
 extern "C" int64_t la_plan_global_capacity(int64_t inserts) { return global_capacity(inserts); }
+#ifdef LA_PROBE_STATS
+extern "C" int la_debug_probe_stats(unsigned long long *out, int reset) {
+    if (cudaMemcpyFromSymbol(out, g_probe_stats, sizeof(unsigned long long) * 8) != cudaSuccess) return -1;
+    if (reset) {
+        unsigned long long z[8] = {};
+        cudaMemcpyToSymbol(g_probe_stats, z, sizeof(z));
+    }
+    return 0;
+}
+#endif
 extern "C" double la_paper_load_factor(int32_t l, int32_t k) { return (double)(l - k + 1) / (double)l; }
 
 // ================================================================================================

@@ -52,9 +52,13 @@ def main():
     want = None
     short = re.sub(r"\(.*", "", kname.replace("void ", ""))
     tmpl = re.search(r"<\(int\)(\d+), \(bool\)(\d)>", kname)
+    tsmall = re.search(r"k_small<\(int\)(\d+)>", kname)
     for n in names:
         if "k_smem" in short and tmpl:
             if n.startswith("_ZN2la6k_smemILi%sELb%s" % (tmpl.group(1), tmpl.group(2))):
+                want = n
+        elif tsmall:
+            if n.startswith("_ZN2la7k_smallILi%sE" % tsmall.group(1)):
                 want = n
         elif short.split("::")[-1] in n:
             want = want or n
