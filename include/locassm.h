@@ -108,12 +108,12 @@ typedef struct {
     int32_t smem_ctas_per_sm;
     int32_t global_rounds;
     int64_t ends_medium;         /* ends routed to the medium (one CTA per SM) kernel             */
-    double ms_smem_medium;       /* device time of the XL + 1- and 2-CTA/SM classes (in ms_smem)   */
+    double ms_smem_medium;       /* summed kernel times of the XL, 2- and 1-CTA/SM classes          */
     int64_t ends_xl;             /* ends whose table lived in the XL class's global scratch        */
     int64_t xl_scratch_bytes;
     /* per table class: 0..4 shared memory (64, 128, 256@3, 256@2, 512 threads), 5 = XL */
     int64_t cls_ends[6], cls_inserts[6], cls_attempts[6], cls_filtered[6];
-    double cls_ms[6];
+    double cls_ms[6];            /* start -> end of each class kernel (classes run concurrently)   */
     /* LA_PROFILE=1 only: per class, summed clock64 cycles of the builders' leader (wait for the
        walker, prefix, clear, filter pass, build pass, link) and of the walker (wait, walk) */
     uint64_t prof_cycles[6][8];
@@ -126,6 +126,19 @@ la_status la_extend(la_ctx *ctx, la_result *out);
 /* Same, but leaves the results on the device only (no device-to-host copy); for device-resident
  * pipelines and the kernel-only benchmark.  Device pointers are returned in *out. */
 la_status la_extend_device(la_ctx *ctx, la_result *out);
+/* Streamed load + extend of a HOST batch (the batched pipeline of Fig 4
+ * L558-563 and the host-to-device staging of P:L480-484).  The batch is cut into up to n_chunks
+ * contiguous contig ranges of ~equal read bytes; chunk i+1's host-to-device copy runs on a second
+ * stream while chunk i is validated, encoded and extended on the context stream, so the copy of a
+ * batch overlaps its extension and device memory holds two chunks of raw input instead of all of it.
+ * batch->mem must be LA_MEM_HOST (pinned memory gives full PCIe bandwidth); n_chunks in 1..4096
+ * (more chunks than contigs is allowed).  Results are identical to la_load_batch + la_extend on the
+ * same batch and are returned like la_extend's (library-owned host memory, valid until the next call
+ * on the context); la_get_stats then reports the work and device time summed over chunks.
+ * Errors: as la_load_batch (an invalid chunk aborts the call with LA_ERR_INVALID_ARG; unlike
+ * la_load_batch, the context's loaded batch is then unspecified until the next la_load_batch). */
+la_status la_extend_streamed(la_ctx *ctx, const la_batch *batch, const la_params *params, int32_t n_chunks,
+                             la_result *out);
 la_status la_get_stats(const la_ctx *ctx, la_stats *out);
 la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
 const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */

@@ -79,7 +79,8 @@ class LocalAssembler:
         if st != L.LA_OK:
             raise L.LocAssmError(st, self._lib.la_last_error(self._ctx).decode())
 
-    def load(self, batch, params=None):
+    @staticmethod
+    def _batch(batch):
         arrs = [batch.contig_seq, batch.contig_off, batch.read_seq, batch.read_qual, batch.read_off,
                 batch.end_read_off]
         ptrs, devs, keep = zip(*[_ptr_and_mem(a) for a in arrs])
@@ -89,6 +90,10 @@ class LocalAssembler:
         n_reads = int(arrs[4].shape[0]) - 1
         b = L.la_batch(L.LA_MEM_DEVICE if devs[0] else L.LA_MEM_HOST, n_contigs, ptrs[0], ptrs[1], n_reads,
                        ptrs[2], ptrs[3], ptrs[4], ptrs[5])
+        return b, keep
+
+    def load(self, batch, params=None):
+        b, keep = self._batch(batch)
         p = _params(params)
         self._check(self._lib.la_load_batch(self._ctx, ctypes.byref(b), ctypes.byref(p)))
         self._keep = keep
@@ -97,6 +102,21 @@ class LocalAssembler:
     def extend(self) -> Result:
         r = L.la_result()
         self._check(self._lib.la_extend(self._ctx, ctypes.byref(r)))
+        return self._result(r)
+
+    def extend_streamed(self, batch, params=None, n_chunks: int = 8) -> Result:
+        """la_extend_streamed: load + extend a HOST batch in n_chunks contig ranges, the host-to-device
+        copy of each chunk overlapping the extension of the previous one."""
+        b, keep = self._batch(batch)
+        p = _params(params)
+        r = L.la_result()
+        self._check(self._lib.la_extend_streamed(self._ctx, ctypes.byref(b), ctypes.byref(p), int(n_chunks),
+                                                 ctypes.byref(r)))
+        del keep
+        return self._result(r)
+
+    @staticmethod
+    def _result(r) -> Result:
         n = int(r.n_ends)
 
         def arr(ptr, count, dtype):

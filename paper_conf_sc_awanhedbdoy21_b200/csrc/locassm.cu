@@ -76,9 +76,18 @@ struct la_ctx {
         g_cur;
     DevBuf lens64, xl_scratch, prof;
     HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
+    // la_extend_streamed: copy stream, double-buffered raw staging (A/B), chunk-ordering events
+    cudaStream_t copy_stream = nullptr;
+    DevBuf st_seq[2], st_qual[2], st_cseq[2], st_coff[2], st_roff[2], st_eoff[2];
+    cudaEvent_t ev_copied[2] = {}, ev_loaded[2] = {};
     int64_t g_attempts = 0;
     cudaEvent_t ev[6] = {};
-    cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] start of XL
+    cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] classes may start
+    cudaEvent_t ev_cls0[N_SMEM_CLASSES + 1] = {};  // start of class c ([N] = XL)
+    // one stream per table class: the persistent class kernels are launched together (largest tables
+    // first) so that the tail of one class overlaps the start of the next; LA_SERIAL_CLASSES=1: one stream
+    cudaStream_t cls_stream[N_SMEM_CLASSES + 1] = {};
+    bool concurrent_classes = true;
     la_stats stats{};
 };
 
@@ -207,7 +216,15 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
+    for (auto &e : ctx->ev_cls0)
+        if (e) cudaEventDestroy(e);
+    for (auto &q : ctx->cls_stream)
+        if (q) cudaStreamDestroy(q);
     for (auto &e : ctx->ev_cls) cudaEventCreate(&e);
+    for (auto &e : ctx->ev_cls0) cudaEventCreate(&e);
+    for (auto &q : ctx->cls_stream)
+        if (cudaStreamCreateWithFlags(&q, cudaStreamNonBlocking) != cudaSuccess) q = nullptr;
+    if (getenv("LA_SERIAL_CLASSES") && atoi(getenv("LA_SERIAL_CLASSES"))) ctx->concurrent_classes = false;
     bool attr_ok = cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         ctx->cls_bytes[N_SMEM_CLASSES - 1]) == cudaSuccess;
     {
@@ -241,6 +258,14 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     ctx->enc.release();
     ctx->spare.release();
+    for (int i = 0; i < 2; ++i) {
+        for (DevBuf *b : {&ctx->st_seq[i], &ctx->st_qual[i], &ctx->st_cseq[i], &ctx->st_coff[i], &ctx->st_roff[i],
+                          &ctx->st_eoff[i]})
+            b->release();
+        if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+        if (ctx->ev_loaded[i]) cudaEventDestroy(ctx->ev_loaded[i]);
+    }
+    if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
     for (DevBuf *b : {&ctx->raw_seq, &ctx->raw_qual, &ctx->raw_coff, &ctx->raw_cseq, &ctx->read_end,
                       &ctx->errw, &ctx->cls, &ctx->out_len, &ctx->out_term, &ctx->out_k, &ctx->out_att,
                       &ctx->walk_buf, &ctx->smem_list, &ctx->smem_key, &ctx->smem_list2, &ctx->smem_key2,
@@ -617,7 +642,14 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         CK(cudaMemsetAsync(prof, 0, 8 * 8 * (N_SMEM_CLASSES + 1), st));
     }
     CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES + 1], st));
+    auto cls_st = [&](int c) -> cudaStream_t {
+        return (ctx->concurrent_classes && ctx->cls_stream[c]) ? ctx->cls_stream[c] : st;
+    };
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c)
+        if (cls_st(c) != st) CK(cudaStreamWaitEvent(cls_st(c), ctx->ev_cls[N_SMEM_CLASSES + 1], 0));
+    CK(cudaEventRecord(ctx->ev_cls0[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));
     if (n_xl > 0) {
+        cudaStream_t st = cls_st(N_SMEM_CLASSES);
         const uint32_t bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
         const uint32_t icap = smem_fixed(dp.W, bytes, 1u).icap;
         const uint32_t stride = xl_stride(xl_rmax, xl_umax, dp.V >= 2, icap);
@@ -634,10 +666,12 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         ctx->stats.ends_xl = n_xl;
         ctx->stats.xl_scratch_bytes = (int64_t)grid * stride;
     }
-    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES], st));   // end of XL
+    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));   // end of XL
     for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
         const int n = ncls[c];
+        CK(cudaEventRecord(ctx->ev_cls0[c], cls_st(c)));
         if (n > 0) {
+            cudaStream_t st = cls_st(c);
             const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm * ctx->cls_ctas[c], n);
             const uint32_t bytes = ctx->cls_bytes[c];
             int32_t *lst = lists + (size_t)c * nE;
@@ -681,9 +715,10 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
 #undef LA_LAUNCH_SMALL
             CKL();
         }
-        if (c == 2) CK(cudaEventRecord(ctx->ev[5], st));   // after the 1- and 2-CTA/SM classes
-        CK(cudaEventRecord(ctx->ev_cls[c], st));   // end of class c
+        CK(cudaEventRecord(ctx->ev_cls[c], cls_st(c)));   // end of class c
     }
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c)   // join
+        if (cls_st(c) != st) CK(cudaStreamWaitEvent(st, ctx->ev_cls[c], 0));
     int n_ovf = 0;
     int n_smem = n_xl;
     for (int c = 0; c < N_SMEM_CLASSES; ++c) n_smem += ncls[c];
@@ -778,29 +813,210 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     ctx->stats.ms_global = ms;
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
     ctx->stats.ms_emit = ms;
-    {
-        cudaEvent_t prev = ctx->ev_cls[N_SMEM_CLASSES + 1];
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {   // start -> end of each class kernel (they may overlap)
         float m = 0;
-        cudaEventElapsedTime(&m, prev, ctx->ev_cls[N_SMEM_CLASSES]);
-        ctx->stats.cls_ms[N_SMEM_CLASSES] = m;
-        prev = ctx->ev_cls[N_SMEM_CLASSES];
-        for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
-            cudaEventElapsedTime(&m, prev, ctx->ev_cls[c]);
-            ctx->stats.cls_ms[c] = m;
-            prev = ctx->ev_cls[c];
-        }
+        cudaEventElapsedTime(&m, ctx->ev_cls0[c], ctx->ev_cls[c]);
+        ctx->stats.cls_ms[c] = m;
     }
     // class counts (host-side tally from the plan counters)
     ctx->stats.ends_by_class[2] = n_smem - n_ovf;
     ctx->stats.ends_by_class[3] = n_glob;
     ctx->stats.ends_by_class[4] = n_ovf;
     ctx->stats.ends_medium = ncls[3] + ncls[4];
-    cudaEventElapsedTime(&ms, ctx->ev[1], ctx->ev[5]);
-    ctx->stats.ms_smem_medium = ms;
+    ctx->stats.ms_smem_medium = ctx->stats.cls_ms[N_SMEM_CLASSES] + ctx->stats.cls_ms[3] + ctx->stats.cls_ms[4];
     return LA_OK;
 }
 
 }  // namespace
 
 extern "C" la_status la_extend(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, true); }
+
+// ---- NEXT N1: streamed load + extend of a host batch (Fig 4) ----------------
+namespace la {
+// in-place rebase of a copied offsets slice: a[i] -= base (the slice's first element)
+__global__ void k_rebase(int64_t *__restrict__ a, int64_t n, int64_t base) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) a[i] -= base;
+}
+__global__ void k_add_i64(const int64_t *__restrict__ a, int64_t n, int64_t add, int64_t *__restrict__ out) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) out[i] = a[i] + add;
+}
+}  // namespace la
+
+extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la_params *params, int32_t n_chunks,
+                                        la_result *out) {
+    if (!ctx || !out) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
+    if (!b || !params) return fail(ctx, LA_ERR_INVALID_ARG, "null batch or params");
+    if (b->mem != LA_MEM_HOST) return fail(ctx, LA_ERR_INVALID_ARG, "la_extend_streamed takes a host batch");
+    if (n_chunks < 1 || n_chunks > 4096) return fail(ctx, LA_ERR_INVALID_ARG, "n_chunks must be in 1..4096");
+    if (b->n_contigs < 0 || b->n_reads < 0) return fail(ctx, LA_ERR_INVALID_ARG, "negative sizes");
+    if (!b->contig_off || !b->read_off || !b->end_read_off)
+        return fail(ctx, LA_ERR_INVALID_ARG, "null offsets array");
+    cudaSetDevice(ctx->device);
+    const int64_t nC = b->n_contigs, nE = 2 * nC, nR = b->n_reads;
+    const int64_t *coff = b->contig_off, *roff = b->read_off, *eoff = b->end_read_off;
+    // the chunking reads offsets at the cut points: check the global invariants it relies on first
+    if (coff[0] != 0 || roff[0] != 0 || eoff[0] != 0) return fail(ctx, LA_ERR_INVALID_ARG, "offsets must start at 0");
+    if (eoff[nE] != nR)
+        return fail(ctx, LA_ERR_INVALID_ARG, "end_read_off[2*n_contigs] (%lld) != n_reads (%lld)",
+                    (long long)eoff[nE], (long long)nR);
+    const int64_t total_bytes = roff[nR];
+    if (total_bytes < 0 || coff[nC] < 0) return fail(ctx, LA_ERR_INVALID_ARG, "negative total length");
+    // contig cuts with ~equal read bytes per chunk (binary search over the monotone prefix); a
+    // non-monotone offsets array is rejected by la_load_batch of the chunk that contains it
+    std::vector<int64_t> cut(1, 0);
+    for (int i = 1; i < n_chunks; ++i) {
+        const int64_t target = total_bytes * i / n_chunks;
+        int64_t lo = cut.back(), hi = nC;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) / 2;
+            const int64_t e = eoff[2 * mid];
+            const int64_t r = (e >= 0 && e <= nR) ? roff[e] : total_bytes;
+            if (r < target) lo = mid + 1; else hi = mid;
+        }
+        if (lo > cut.back() && lo < nC) cut.push_back(lo);
+    }
+    cut.push_back(nC);
+    const int nchunk = (int)cut.size() - 1;
+    if (!ctx->copy_stream) {
+        CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+        for (int i = 0; i < 2; ++i) {
+            CK(cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&ctx->ev_loaded[i], cudaEventDisableTiming));
+        }
+    }
+    cudaStream_t cs = ctx->copy_stream, st = ctx->stream;
+    const int W = std::max(params->max_walk_len, 1);
+    // combined host results (pinned, grow-only): the extension bytes are bounded by W per end
+    CK(grow_host(ctx->h_ext_off, (nE + 1) * 8));
+    CK(grow_host(ctx->h_ext_seq, nE * (int64_t)W + 16));
+    CK(grow_host(ctx->h_term, nE + 16));
+    CK(grow_host(ctx->h_k, nE + 16));
+    CK(grow_host(ctx->h_att, nE + 16));
+    int64_t *h_off = (int64_t *)ctx->h_ext_off.p;
+    h_off[0] = 0;
+    // chunk c: contigs [cut[c], cut[c+1]) -> ends, reads, bytes (all contiguous ranges)
+    struct Chunk { int64_t c0, c1, r0, r1, b0, b1, s0, s1; };
+    std::vector<Chunk> chunks(nchunk);
+    for (int c = 0; c < nchunk; ++c) {   // cut points must be ordered (the chunks check the rest)
+        Chunk &k = chunks[c];
+        k.c0 = cut[c]; k.c1 = cut[c + 1];
+        k.r0 = eoff[2 * k.c0]; k.r1 = eoff[2 * k.c1];
+        if (k.r0 < 0 || k.r1 < k.r0 || k.r1 > nR)
+            return fail(ctx, LA_ERR_INVALID_ARG, "offsets are not non-decreasing");
+        k.b0 = roff[k.r0]; k.b1 = roff[k.r1];
+        k.s0 = coff[k.c0]; k.s1 = coff[k.c1];
+        if (k.b0 < 0 || k.b1 < k.b0 || k.s0 < 0 || k.s1 < k.s0)
+            return fail(ctx, LA_ERR_INVALID_ARG, "offsets are not non-decreasing");
+    }
+    auto chunk = [&](int c) { return chunks[c]; };
+    auto enqueue_copy = [&](int c) -> la_status {
+        const int i = c & 1;
+        const Chunk k = chunk(c);
+        const int64_t nc = k.c1 - k.c0, nr = k.r1 - k.r0;
+        CK(grow(ctx->st_seq[i], k.b1 - k.b0 + 16));
+        CK(grow(ctx->st_qual[i], k.b1 - k.b0 + 16));
+        CK(grow(ctx->st_cseq[i], k.s1 - k.s0 + 16));
+        CK(grow(ctx->st_coff[i], (nc + 1) * 8));
+        CK(grow(ctx->st_roff[i], (nr + 1) * 8));
+        CK(grow(ctx->st_eoff[i], (2 * nc + 1) * 8));
+        if (c >= 2) CK(cudaStreamWaitEvent(cs, ctx->ev_loaded[i], 0));   // chunk c-2 is encoded: buffer free
+        if (k.b1 > k.b0) {
+            if (!b->read_seq || !b->read_qual) return fail(ctx, LA_ERR_INVALID_ARG, "null sequence pointer");
+            CK(cudaMemcpyAsync(ctx->st_seq[i].p, b->read_seq + k.b0, k.b1 - k.b0, cudaMemcpyHostToDevice, cs));
+            CK(cudaMemcpyAsync(ctx->st_qual[i].p, b->read_qual + k.b0, k.b1 - k.b0, cudaMemcpyHostToDevice, cs));
+        }
+        if (k.s1 > k.s0) {
+            if (!b->contig_seq) return fail(ctx, LA_ERR_INVALID_ARG, "null sequence pointer");
+            CK(cudaMemcpyAsync(ctx->st_cseq[i].p, b->contig_seq + k.s0, k.s1 - k.s0, cudaMemcpyHostToDevice, cs));
+        }
+        CK(cudaMemcpyAsync(ctx->st_coff[i].p, coff + k.c0, (nc + 1) * 8, cudaMemcpyHostToDevice, cs));
+        CK(cudaMemcpyAsync(ctx->st_roff[i].p, roff + k.r0, (nr + 1) * 8, cudaMemcpyHostToDevice, cs));
+        CK(cudaMemcpyAsync(ctx->st_eoff[i].p, eoff + 2 * k.c0, (2 * nc + 1) * 8, cudaMemcpyHostToDevice, cs));
+        CK(cudaEventRecord(ctx->ev_copied[i], cs));
+        return LA_OK;
+    };
+    la_status s;
+    if ((s = enqueue_copy(0))) return s;
+    if (nchunk > 1 && (s = enqueue_copy(1))) return s;
+    la_stats acc{};
+    int64_t bases = 0;
+    for (int c = 0; c < nchunk; ++c) {
+        const int i = c & 1;
+        const Chunk k = chunk(c);
+        const int64_t nc = k.c1 - k.c0, nr = k.r1 - k.r0;
+        CK(cudaStreamWaitEvent(st, ctx->ev_copied[i], 0));
+        k_rebase<<<blocks(nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_coff[i]), nc + 1, k.s0);
+        k_rebase<<<blocks(nr + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_roff[i]), nr + 1, k.b0);
+        k_rebase<<<blocks(2 * nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_eoff[i]), 2 * nc + 1, k.r0);
+        CK(cudaGetLastError());
+        la_batch sub{};
+        sub.mem = LA_MEM_DEVICE;
+        sub.n_contigs = (int32_t)nc;
+        sub.contig_seq = P<char>(ctx->st_cseq[i]);
+        sub.contig_off = P<int64_t>(ctx->st_coff[i]);
+        sub.n_reads = nr;
+        sub.read_seq = P<char>(ctx->st_seq[i]);
+        sub.read_qual = P<char>(ctx->st_qual[i]);
+        sub.read_off = P<int64_t>(ctx->st_roff[i]);
+        sub.end_read_off = P<int64_t>(ctx->st_eoff[i]);
+        if ((s = la_load_batch(ctx, &sub, params))) return s;
+        CK(cudaEventRecord(ctx->ev_loaded[i], st));   // staging buffer i may be refilled
+        if (c + 2 < nchunk && (s = enqueue_copy(c + 2))) return s;
+        la_result r{};
+        if ((s = extend_impl(ctx, &r, false))) return s;
+        const int64_t ne = 2 * nc, nb = ctx->stats.ext_bases;
+        // results of this chunk -> the combined host buffers (device-side rebase of ext_off)
+        CK(grow(ctx->lens64, (ne + 1) * 8));
+        k_add_i64<<<blocks(ne + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->ext_off), ne + 1, bases, P<int64_t>(ctx->lens64));
+        CK(cudaGetLastError());
+        const int64_t e0 = 2 * k.c0;
+        CK(cudaMemcpyAsync(h_off + e0 + 1, P<int64_t>(ctx->lens64) + 1, ne * 8, cudaMemcpyDeviceToHost, st));
+        if (nb) CK(cudaMemcpyAsync((char *)ctx->h_ext_seq.p + bases, ctx->ext_seq.p, nb, cudaMemcpyDeviceToHost, st));
+        if (ne) {
+            CK(cudaMemcpyAsync((uint8_t *)ctx->h_term.p + e0, ctx->out_term.p, ne, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync((uint8_t *)ctx->h_k.p + e0, ctx->out_k.p, ne, cudaMemcpyDeviceToHost, st));
+            CK(cudaMemcpyAsync((uint8_t *)ctx->h_att.p + e0, ctx->out_att.p, ne, cudaMemcpyDeviceToHost, st));
+        }
+        bases += nb;
+        // accumulate the work and device-time counters over chunks
+        const la_stats &x = ctx->stats;
+        acc.ms_total += x.ms_total;
+        acc.ms_smem += x.ms_smem;
+        acc.ms_global += x.ms_global;
+        acc.ms_emit += x.ms_emit;
+        acc.inserts += x.inserts;
+        acc.inserts_smem += x.inserts_smem;
+        acc.walk_steps += x.walk_steps;
+        acc.attempts += x.attempts;
+        acc.ext_bases += x.ext_bases;
+        for (int q = 0; q < 5; ++q) acc.ends_by_class[q] += x.ends_by_class[q];
+        acc.kernel_launches += x.kernel_launches + 4;   // + the rebase / offset kernels
+        acc.global_rounds += x.global_rounds;
+        acc.ends_medium += x.ends_medium;
+        acc.ms_smem_medium += x.ms_smem_medium;
+        acc.ends_xl += x.ends_xl;
+        acc.xl_scratch_bytes = std::max(acc.xl_scratch_bytes, x.xl_scratch_bytes);
+        for (int q = 0; q < 6; ++q) {
+            acc.cls_ends[q] += x.cls_ends[q];
+            acc.cls_inserts[q] += x.cls_inserts[q];
+            acc.cls_attempts[q] += x.cls_attempts[q];
+            acc.cls_filtered[q] += x.cls_filtered[q];
+            acc.cls_ms[q] += x.cls_ms[q];
+        }
+        acc.smem_bytes_per_cta = x.smem_bytes_per_cta;
+        acc.smem_ctas_per_sm = x.smem_ctas_per_sm;
+    }
+    CK(cudaStreamSynchronize(st));
+    ctx->stats = acc;
+    out->n_ends = nE;
+    out->ext_off = h_off;
+    out->ext_seq = (const char *)ctx->h_ext_seq.p;
+    out->term = (const uint8_t *)ctx->h_term.p;
+    out->k_used = (const uint8_t *)ctx->h_k.p;
+    out->n_attempts = (const uint8_t *)ctx->h_att.p;
+    return LA_OK;
+}
 extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, false); }

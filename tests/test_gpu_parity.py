@@ -194,3 +194,49 @@ def test_state_error_before_load():
     with LocalAssembler(0) as la:
         with pytest.raises(LocAssmError, match="STATE"):
             la.extend()
+
+
+@pytest.fixture(scope="module")
+def c2_ref(orc):
+    b = cached_batch("C2", scale=0.03)
+    return b, orc.extend(b, P0)
+
+
+@pytest.mark.parametrize("n_chunks", [1, 3, 8, 4000])
+def test_streamed_matches_oracle(LA, c2_ref, n_chunks):
+    """la_extend_streamed (NEXT N1): chunked host batch, copies overlapped with extension — every end
+    bit-exact against the oracle, work counters summed over chunks; 4000 chunks > contigs."""
+    b, ref = c2_ref
+    r = LA.extend_streamed(b, P0, n_chunks)
+    st = LA.stats()
+    assert r.ext_list() == ref["ext"]
+    for f in ("term", "k_used", "n_attempts"):
+        assert np.array_equal(getattr(r, f), ref[f]), f
+    assert st["inserts"] == int(ref["inserts"].sum())
+    assert st["walk_steps"] == int(ref["walk_steps"].sum())
+    # the context stays usable for the ordinary load + extend path
+    assert LA.load(b.select_contigs(np.arange(20)), P0).extend().n_ends == 40
+
+
+def test_streamed_edge_cases(LA, orc):
+    from paper_conf_sc_awanhedbdoy21_b200._lib import LocAssmError
+    import torch
+    empty = C.Batch.from_lists([], [])
+    assert LA.extend_streamed(empty, P0, 4).n_ends == 0
+    small = C.Batch.from_lists(["ACGT" * 20, "A"], [[("N" * 150, "I" * 150)], [], [], []])
+    ref = orc.extend(small, P0)
+    r = LA.extend_streamed(small, P0, 2)
+    assert r.ext_list() == ref["ext"] and np.array_equal(r.term, ref["term"])
+    with pytest.raises(LocAssmError, match="n_chunks"):
+        LA.extend_streamed(small, P0, 0)
+    bad = C.Batch.from_lists(["ACGT" * 10, "ACGTX" * 10], [[], [], [], []])
+    with pytest.raises(LocAssmError, match="INVALID_ARG"):
+        LA.extend_streamed(bad, P0, 2)
+
+    class DevBatch:
+        pass
+    d = DevBatch()
+    for f in ("contig_seq", "contig_off", "read_seq", "read_qual", "read_off", "end_read_off"):
+        setattr(d, f, torch.from_numpy(getattr(small, f)).cuda())
+    with pytest.raises(LocAssmError, match="host batch"):
+        LA.extend_streamed(d, P0, 2)
