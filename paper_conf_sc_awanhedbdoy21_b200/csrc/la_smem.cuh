@@ -328,9 +328,13 @@ __device__ __forceinline__ void votes_of(const TabCtx &T, uint32_t s, uint32_t l
     }
 }
 
+// Inline-key tables probe linearly from an even slot, so that a probe round can test the slot pair
+// (s, s+1) with two adjacent 16 B loads (cap is even).
+__device__ __forceinline__ uint32_t slot0_inl(uint64_t h, uint32_t cap) { return slot_of(h, cap) & ~1u; }
+
 template <bool INL, int NW>
 __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> &K, uint64_t h) {
-    uint32_t s = slot_of(h, T.cap);
+    uint32_t s = INL ? slot0_inl(h, T.cap) : slot_of(h, T.cap);
     if (INL) {
         uint64_t a, b;
         inline_form(K, T.KW, a, b);
@@ -489,19 +493,16 @@ struct PosV {            // one lane's position
 
 __device__ __forceinline__ uint64_t nmask_word(uint64_t q) { return q & (q >> 1) & 0x5555555555555555ull; }
 
-// position p of read row (R, Q); has_n: the read contains an N (rflag)
-__device__ __forceinline__ PosV pos_value(const uint64_t *R, const uint64_t *Q, int p, int k, int KW, int SW,
-                                          bool has_n) {
+// position p of read row (R, Q); has_n: the read contains an N (rflag); m0, m1: masks of the k-mer's
+// bits in its two words (hoisted out of the position loop)
+__device__ __forceinline__ PosV pos_value(const uint64_t *R, const uint64_t *Q, int p, int k, int SW, bool has_n,
+                                          uint64_t m0, uint64_t m1) {
     PosV v;
     const int q = p >> 5, s = (p & 31) << 1;
     const int q2 = min(q + 2, SW - 1);   // word q+2 is only needed when the window reaches it
     const uint64_t r0 = R[q], r1 = R[q + 1], r2 = R[q2];
-    const int b1 = 2 * k - 64;           // bits of word 1 (<= 0: k <= 32)
-    const uint64_t m0 = b1 >= 0 ? ~0ull : (~0ull << (64 - 2 * k));
-    const uint64_t m1 = b1 > 0 ? (~0ull << (64 - b1)) : 0ull;
     v.K.w[0] = funnel64(r0, r1, s) & m0;
     v.K.w[1] = funnel64(r1, r2, s) & m1;
-    (void)KW;
     const int i = p + k, wi = i >> 5, d = wi - q;   // following base, word q+d (d in 0..2)
     const uint64_t rw = d == 0 ? r0 : (d == 1 ? r1 : r2);
     const int sh = 62 - ((i & 31) << 1);
@@ -516,16 +517,25 @@ __device__ __forceinline__ PosV pos_value(const uint64_t *R, const uint64_t *Q, 
     return v;
 }
 
+__device__ __forceinline__ void kmer_masks(int k, uint64_t &m0, uint64_t &m1) {
+    const int b1 = 2 * k - 64;   // bits of word 1 (<= 0: k <= 32)
+    m0 = b1 >= 0 ? ~0ull : (~0ull << (64 - 2 * k));
+    m1 = b1 > 0 ? (~0ull << (64 - b1)) : 0ull;
+}
+
 // f(act, v): act = this lane has a position this iteration (warp-uniform call).
 template <typename F>
 __device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
                                                const uint8_t *__restrict__ rflag, const uint32_t *pref,
                                                long long r0, int r, int SW, int k, int KW, int wid, int nwarps,
                                                int lane, const volatile int *stop, F &&f) {
+    (void)KW;
     const uint32_t total = pref[r];
     const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
     const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
     if (wb >= we) return;
+    uint64_t m0, m1;
+    kmer_masks(k, m0, m1);
     uint32_t g = wb + lane;
     int j;
     {   // read j with pref[j] <= g < pref[j+1]
@@ -537,16 +547,26 @@ __device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq
         }
         j = lo;
     }
+    // the lane's current read: position range [pj0, pj1), rows R / Q, has-N flag
+    uint32_t pj0 = pref[j], pj1 = pref[j + 1];
+    const uint64_t *R = rseq + (r0 + j) * SW, *Q = rqc + (r0 + j) * SW;
+    bool flag = rflag[r0 + j] != 0;
     for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
         if (__shfl_sync(0xffffffffu, *stop, 0)) return;
         const bool act = g < we;
         PosV v;
         v.vote = false;
         if (act) {
-            uint32_t pj = pref[j + 1];
-            while (pj <= g) pj = pref[++j + 1];   // crossed into a later read (skips reads without positions)
-            const long long rid = r0 + j;
-            v = pos_value(rseq + rid * SW, rqc + rid * SW, (int)(g - pref[j]), k, KW, SW, rflag[rid] != 0);
+            if (g >= pj1) {   // crossed into a later read (skips reads without positions)
+                do {
+                    pj0 = pj1;
+                    pj1 = pref[++j + 1];
+                } while (g >= pj1);
+                R = rseq + (r0 + j) * SW;
+                Q = rqc + (r0 + j) * SW;
+                flag = rflag[r0 + j] != 0;
+            }
+            v = pos_value(R, Q, (int)(g - pj0), k, SW, flag, m0, m1);
         }
         f(act && v.vote, v);
     }
@@ -630,13 +650,35 @@ __device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, con
 }
 
 // Convergent insert of the lanes with `want` (Alg 1 line 5 + the vote): every probe round
-// is entered by the whole warp; claims are counted once per warp.
+// is entered by the whole warp and tests a slot pair (s, s+1); claims are counted once per warp.
+// One slot of a round: 0 = resolved (found or claimed), 1 = occupied by another key, 2 = gave up
+// (overflow flagged), 3 = lost the claim race to another key (re-probe from this slot's successor).
+template <bool GT>
+__device__ __forceinline__ int probe_slot(const TabCtx &T, uint32_t s, uint64_t x, uint64_t y, uint64_t a, uint64_t bb,
+                                          bool &claimed, volatile int *ovf) {
+    if (y == 0) {   // looks empty: the CAS claims it or returns its true content
+        if (*ovf) return 2;
+        cas128<GT>((void *)&T.keys[2 * (size_t)s], 0ull, 0ull, a, bb, x, y);
+        if (y == 0) {
+            claimed = true;
+            return 0;
+        }
+        if (y == bb && x != a) x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
+        return (x == a && y == bb) ? 0 : 3;
+    }
+    // a 16 B load is not single-copy atomic: if it raced with the claiming CAS, word 0 may be stale —
+    // re-read it (a slot never changes once claimed)
+    if (y == bb && x != a) x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
+    return (x == a && y == bb) ? 0 : 1;
+}
+
 template <bool GT>
 __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const PosV &v, uint64_t h, int lane,
                                             int *nclaim, int claim_limit, volatile int *ovf) {
-    uint32_t s = slot_of(h, T.cap);
+    uint32_t s = slot0_inl(h, T.cap);
     const uint64_t a = v.K.w[0], bb = ~(T.KW >= 2 ? v.K.w[1] : 0ull);
     bool pend = want, found = false;
+    uint32_t hit = 0;
 #ifdef LA_PROBE_STATS
     { const unsigned m = __ballot_sync(0xffffffffu, want); if (lane == 0) { LA_PSTAT(0, 1); LA_PSTAT(2, __popc(m)); } }
 #endif
@@ -644,30 +686,29 @@ __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const Po
         if (lane == 0) LA_PSTAT(1, 1);
         bool claimed = false;
         if (pend) {
-            uint64_t x, y;
-            ld128v<GT>(&T.keys[2 * (size_t)s], x, y);
-            if (y == 0) {   // looks empty: the CAS claims it or returns its true content
-                if (*ovf) {
-                    pend = false;
-                } else {
-                    cas128<GT>((void *)&T.keys[2 * (size_t)s], 0ull, 0ull, a, bb, x, y);
-                    if (y == 0) {
-                        claimed = true;
-                        x = a;
-                        y = bb;
-                    }
-                }
-            } else if (y == bb && x != a) {
-                // a 16 B load is not single-copy atomic: if it raced with the claiming CAS, word 0 may
-                // be stale — re-read it (a slot never changes once claimed)
-                x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
-            }
-            if (pend) {
-                if (x == a && y == bb) {
+            uint64_t x0, y0, x1, y1;
+            const uint32_t s1 = s + 1 == T.cap ? 0 : s + 1;   // s is even except after a lost claim race
+            ld128v<GT>(&T.keys[2 * (size_t)s], x0, y0);
+            ld128v<GT>(&T.keys[2 * (size_t)s1], x1, y1);
+            int st = probe_slot<GT>(T, s, x0, y0, a, bb, claimed, ovf);
+            if (st == 0) {
+                hit = s;
+                pend = false;
+                found = true;
+            } else if (st == 2) {
+                pend = false;
+            } else if (st == 3) {
+                s = s1;   // the slot pair loaded before the lost race may be stale: next round
+            } else {
+                st = probe_slot<GT>(T, s1, x1, y1, a, bb, claimed, ovf);
+                if (st == 0) {
+                    hit = s1;
                     pend = false;
                     found = true;
+                } else if (st == 2) {
+                    pend = false;
                 } else {
-                    s = (s + 1 == T.cap) ? 0 : s + 1;
+                    s = s1 + 1 == T.cap ? 0 : s1 + 1;
                 }
             }
         }
@@ -678,13 +719,13 @@ __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const Po
             if (atomicAdd(nclaim, n) + n > claim_limit) *ovf = 1;
         }
     }
-    if (found) vote_add<GT>(T, s, v.nb, v.hi, ovf);
+    if (found) vote_add<GT>(T, hit, v.nb, v.hi, ovf);
 }
 
-// Convergent lookup (no insert): slot of K or NONE.
+// Convergent lookup (no insert): slot of K or NONE; slot pairs as in warp_insert.
 template <bool GT>
 __device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, const KmerN<2> &K, uint64_t h) {
-    uint32_t s = slot_of(h, T.cap), res = NONE;
+    uint32_t s = slot0_inl(h, T.cap), res = NONE;
     const uint64_t a = K.w[0], bb = ~(T.KW >= 2 ? K.w[1] : 0ull);
     bool pend = want;
     uint32_t n = 0;
@@ -694,16 +735,23 @@ __device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, cons
     while (__any_sync(0xffffffffu, pend)) {
         if ((threadIdx.x & 31) == 0) LA_PSTAT(5, 1);
         if (pend) {
-            uint64_t x, y;
-            ld128v<GT>(&T.keys[2 * (size_t)s], x, y);
-            if (y == 0) {
+            uint64_t x0, y0, x1, y1;
+            ld128v<GT>(&T.keys[2 * (size_t)s], x0, y0);
+            ld128v<GT>(&T.keys[2 * (size_t)s + 2], x1, y1);   // s even, cap even: s+1 < cap
+            if (y0 == 0) {
                 pend = false;
-            } else if (x == a && y == bb) {
+            } else if (x0 == a && y0 == bb) {
                 pend = false;
                 res = s;
+            } else if (y1 == 0) {
+                pend = false;
+            } else if (x1 == a && y1 == bb) {
+                pend = false;
+                res = s + 1;
             } else {
-                s = (s + 1 == T.cap) ? 0 : s + 1;
-                if (++n >= T.cap) pend = false;
+                s = s + 2 == T.cap ? 0 : s + 2;
+                n += 2;
+                if (n >= T.cap) pend = false;
             }
         }
     }
