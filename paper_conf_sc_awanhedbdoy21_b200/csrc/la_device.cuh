@@ -129,23 +129,20 @@ __device__ __forceinline__ uint32_t get2(const uint64_t *R, int i) {
 }
 
 // Reading #1: two-tier vote rule on exact integer counts.  Returns 0..3 (base), CODE_FORK or
-// CODE_DEADEND.
+// CODE_DEADEND.  Branch-free (selects only): it runs slot-parallel in the link pass, where data-
+// dependent branches split the warp.
 __device__ __forceinline__ int ext_rule(const uint32_t lo[4], const uint32_t hi[4], int V, int F) {
-    uint64_t H = (uint64_t)hi[0] + hi[1] + hi[2] + hi[3];
-    uint64_t L = (uint64_t)lo[0] + lo[1] + lo[2] + lo[3];
-    int n = 0, pick = 0;
+    const uint64_t H = (uint64_t)hi[0] + hi[1] + hi[2] + hi[3];
+    const uint64_t L = (uint64_t)lo[0] + lo[1] + lo[2] + lo[3];
+    uint32_t mh = 0, ml = 0;
 #pragma unroll
-    for (int b = 0; b < 4; ++b)
-        if (hi[b] >= (uint32_t)V && 100ull * hi[b] >= (uint64_t)F * H) { ++n; pick = b; }
-    if (n == 1) return pick;
-    if (n >= 2) return CODE_FORK;
-    n = 0;
-#pragma unroll
-    for (int b = 0; b < 4; ++b)
-        if (lo[b] >= (uint32_t)V && 100ull * lo[b] >= (uint64_t)F * L) { ++n; pick = b; }
-    if (n == 1) return pick;
-    if (n >= 2) return CODE_FORK;
-    return CODE_DEADEND;
+    for (int b = 0; b < 4; ++b) {
+        mh |= (hi[b] >= (uint32_t)V && 100ull * hi[b] >= (uint64_t)F * H) ? (1u << b) : 0u;
+        ml |= (lo[b] >= (uint32_t)V && 100ull * lo[b] >= (uint64_t)F * L) ? (1u << b) : 0u;
+    }
+    const uint32_t m = mh ? mh : ml;   // the high tier decides when it has a candidate
+    const int one = __ffs(m) - 1;
+    return m == 0 ? CODE_DEADEND : ((m & (m - 1)) ? CODE_FORK : one);
 }
 
 // The k up/down-shift rule (readings #8, #10).  Returns true when the end is done,

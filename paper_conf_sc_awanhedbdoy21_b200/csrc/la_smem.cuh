@@ -552,7 +552,7 @@ __device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq
     const uint64_t *R = rseq + (r0 + j) * SW, *Q = rqc + (r0 + j) * SW;
     bool flag = rflag[r0 + j] != 0;
     for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
-        if (__shfl_sync(0xffffffffu, *stop, 0)) return;
+        if (((base - wb) & 127u) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;   // every 4th iteration
         const bool act = g < we;
         PosV v;
         v.vote = false;
@@ -857,6 +857,21 @@ __device__ __forceinline__ void read_prefix(BuildCtl &B, EndSlot &E, uint32_t *p
     }
 }
 
+// Position of the n-th (0-based) set bit of m (n < popc(m)): popc bisection, selects only (__fns is
+// a software loop on sm_100a: 6% of the small-class kernel's instructions, ncu r01).
+__device__ __forceinline__ uint32_t nth_set_bit(uint32_t m, uint32_t n) {
+    uint32_t pos = 0;
+#pragma unroll
+    for (int w = 16; w >= 1; w >>= 1) {
+        const uint32_t c = __popc(m & ((1u << w) - 1u));
+        const bool up = n >= c;
+        n = up ? n - c : n;
+        pos = up ? pos + w : pos;
+        m = up ? m >> w : m;
+    }
+    return pos;
+}
+
 // Slot-parallel pass after the build: ext(lo, hi) (reading #1, a5) and, for a base, the successor
 // k-mer's slot (next_kmer, Alg 2 line 15) -> info[s] = next << 4 | code.
 __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
@@ -989,12 +1004,12 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             }
             const int n = __popc(m), tot = qn + n;
             const int t = lane - qn;   // rank (in m) of the new slot this lane takes
-            const uint32_t mine = lane < qn ? qs : (t < n ? base + __fns(m, 0, t + 1) : 0u);
+            const uint32_t mine = lane < qn ? qs : (t < n ? base + nth_set_bit(m, (uint32_t)t) : 0u);
             if (tot >= 32 || (!more && tot > 0)) {
                 link_batch(lane < tot, mine);
                 const int t2 = 32 - qn + lane;   // leftover ranks 32-qn .. n-1 -> lanes 0..
                 qn = tot > 32 ? tot - 32 : 0;
-                qs = lane < qn ? base + __fns(m, 0, t2 + 1) : 0u;
+                qs = lane < qn ? base + nth_set_bit(m, (uint32_t)t2) : 0u;
             } else {
                 qs = mine;
                 qn = tot;

@@ -10,4 +10,4 @@ import json; d=json.load(open('gpurun_out/bench_quick.json'))
 print('ms/step', d['ms_per_step'], 'value', d['value'], 'frac', d['roofline']['frac'])
 for k,v in d['work']['classes'].items(): print(k, v)
 "
-if [ -n "$PHASE" ]; then timeout 600 python tools/phase_profile.py > gpurun_out/phase.json 2> gpurun_out/phase.err; fi
+if [ -n "$PHASE" ]; then LA_SERIAL_CLASSES=1 timeout 600 python tools/phase_profile.py > gpurun_out/phase.json 2> gpurun_out/phase.err; fi
