@@ -78,7 +78,7 @@ __host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, 
 }
 
 struct SmemTab {
-    uint32_t off_pref, off_b1, off_b2, off_keys, off_cnts, cap, mwords;
+    uint32_t off_pref, off_b1, off_b2, off_keys, off_cnts, off_list, cap, mwords;
 };
 
 __host__ __device__ __forceinline__ uint32_t pref_bytes(int r) { return (((uint32_t)r + 1u) * 4u + 15u) & ~15u; }
@@ -100,7 +100,7 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
     const uint32_t sb = gt ? 0u : stage_bytes(r, SW);   // shared-memory tables: reads staged first
     const uint32_t pb = pref_bytes(r) + sb;
     const uint32_t tab = F.tab_bytes > pb ? F.tab_bytes - pb : 0u;
-    const uint32_t per_slot = kbytes + cnt_bytes(gt);
+    const uint32_t per_slot = kbytes + cnt_bytes(gt) + 2u;   // key + counters + claim-list entry (u16)
     uint32_t cap_nf = tab / per_slot;
     if (cap_nf > F.icap) cap_nf = F.icap;
     cap_nf &= ~1u;
@@ -137,6 +137,7 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
     T.cap = cap;
     T.mwords = mwords;
     T.off_cnts = T.off_keys + cap * kbytes;
+    T.off_list = T.off_cnts + cap * cnt_bytes(gt);
     return T;
 }
 
@@ -184,7 +185,7 @@ __host__ __device__ __forceinline__ uint32_t xl_needed_cap(int64_t r, int64_t U,
 __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_max, bool filter, uint32_t icap) {
     uint32_t cap = xl_needed_cap(r_max, U_max, filter);
     if (cap > icap) cap = icap;
-    return (pref_bytes((int)r_max) + 32u + cap * (16u + cnt_bytes(true)) + 255u) & ~255u;
+    return (pref_bytes((int)r_max) + 32u + cap * (16u + cnt_bytes(true) + 2u) + 255u) & ~255u;
 }
 
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
@@ -292,7 +293,8 @@ __device__ __forceinline__ void inline_form(const KmerN<NW> &K, int KW, uint64_t
 
 struct TabCtx {   // what a table operation needs
     uint64_t *keys;
-    uint32_t *c32;   // per slot: word 0 = lo[4] (8 bits each), word 1 = hi[4]
+    uint32_t *c32;   // per slot: word 0 = low-only votes[4] (8 bits each), word 1 = high votes[4]
+    uint16_t *list;  // claimed slots in claim order (inline keys): the link pass visits only these
     uint32_t cap;
     const uint64_t *rseq;   // packed reads (global), for REF-format key verification
     int SW, k, KW;
@@ -713,10 +715,17 @@ __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const Po
             }
         }
         const unsigned cm = __ballot_sync(0xffffffffu, claimed);
-        if (cm && lane == __ffs(cm) - 1) {
-            const int n = __popc(cm);
-            LA_PSTAT(3, n);
-            if (atomicAdd(nclaim, n) + n > claim_limit) *ovf = 1;
+        if (cm) {
+            const int n = __popc(cm), leader = __ffs(cm) - 1;
+            int first = 0;
+            if (lane == leader) {
+                LA_PSTAT(3, n);
+                first = atomicAdd(nclaim, n);
+                if (first + n > claim_limit) *ovf = 1;
+            }
+            first = __shfl_sync(0xffffffffu, first, leader);
+            // claims <= cap always (a claim takes an empty slot), so the list cannot overflow
+            if (claimed) T.list[first + __popc(cm & ((1u << lane) - 1u))] = (uint16_t)hit;
         }
     }
     if (found) vote_add<GT>(T, hit, v.nb, v.hi, ovf);
@@ -857,21 +866,6 @@ __device__ __forceinline__ void read_prefix(BuildCtl &B, EndSlot &E, uint32_t *p
     }
 }
 
-// Position of the n-th (0-based) set bit of m (n < popc(m)): popc bisection, selects only (__fns is
-// a software loop on sm_100a: 6% of the small-class kernel's instructions, ncu r01).
-__device__ __forceinline__ uint32_t nth_set_bit(uint32_t m, uint32_t n) {
-    uint32_t pos = 0;
-#pragma unroll
-    for (int w = 16; w >= 1; w >>= 1) {
-        const uint32_t c = __popc(m & ((1u << w) - 1u));
-        const bool up = n >= c;
-        n = up ? n - c : n;
-        pos = up ? pos + w : pos;
-        m = up ? m >> w : m;
-    }
-    return pos;
-}
-
 // Slot-parallel pass after the build: ext(lo, hi) (reading #1, a5) and, for a base, the successor
 // k-mer's slot (next_kmer, Alg 2 line 15) -> info[s] = next << 4 | code.
 __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
@@ -963,9 +957,8 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
 #endif
     // ---- ext rule + successor links (a5) into the end's info buffer ----
     if (INL) {
-        // Occupied slots (~30% of the table) are compacted into full warps first: each warp scans
-        // its chunks of 32 slots and queues the occupied ones in a one-slot-per-lane register queue;
-        // every full queue (and the final partial one) is linked with all lanes busy.
+        // Only occupied slots (~30% of the table) are visited: warp_insert appends every claimed slot
+        // to the claim list, so the warps take 32 list entries at a time with all lanes busy.
         auto link_batch = [&](bool has, uint32_t s) {
             KmerN<2> K;
             K.w[0] = K.w[1] = 0;
@@ -982,39 +975,11 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             const uint32_t t = warp_lookup<GT>(T, has && code < 4, K, hash_kmer(K, KW));
             if (has) info[s] = link_info(code, t);
         };
-#ifndef LA_LINK_COMPACT
-#define LA_LINK_COMPACT 1
-#endif
-        if (!LA_LINK_COMPACT) {
-            for (uint32_t base = (uint32_t)wid * 32u; base < T.cap; base += (uint32_t)NB) {
-                const uint32_t s = base + lane;
-                link_batch(s < T.cap && ((const ulonglong2 *)T.keys)[min(s, T.cap - 1)].y != 0, s);
-            }
-        }
-        uint32_t qs = 0;
-        int qn = 0;
-        for (uint32_t base = (uint32_t)wid * 32u; LA_LINK_COMPACT; base += (uint32_t)NB) {
-            const bool more = base < T.cap;   // warp-uniform
-            uint32_t m = 0;
-            if (more) {
-                const uint32_t s = base + lane;
-                bool occ = false;
-                if (s < T.cap) occ = ((const ulonglong2 *)T.keys)[s].y != 0;
-                m = __ballot_sync(0xffffffffu, occ);
-            }
-            const int n = __popc(m), tot = qn + n;
-            const int t = lane - qn;   // rank (in m) of the new slot this lane takes
-            const uint32_t mine = lane < qn ? qs : (t < n ? base + nth_set_bit(m, (uint32_t)t) : 0u);
-            if (tot >= 32 || (!more && tot > 0)) {
-                link_batch(lane < tot, mine);
-                const int t2 = 32 - qn + lane;   // leftover ranks 32-qn .. n-1 -> lanes 0..
-                qn = tot > 32 ? tot - 32 : 0;
-                qs = lane < qn ? base + nth_set_bit(m, (uint32_t)t2) : 0u;
-            } else {
-                qs = mine;
-                qn = tot;
-            }
-            if (!more) break;
+        // the claimed slots, in claim order (warp_insert), all lanes busy
+        const uint32_t nocc = min((uint32_t)B.nclaim, T.cap);
+        for (uint32_t base = (uint32_t)wid * 32u; base < nocc; base += (uint32_t)NB) {
+            const uint32_t i = base + lane;
+            link_batch(i < nocc, i < nocc ? (uint32_t)T.list[i] : 0u);
         }
     } else {
         constexpr int NW = MAX_KW;
@@ -1290,6 +1255,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             if (TB.cap > need) {
                 TB.cap = (need + 1u) & ~1u;
                 TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
+                TB.off_list = TB.off_cnts + TB.cap * cnt_bytes(true);
             }
         }
         bool ovf = no_room || TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
@@ -1301,6 +1267,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             TabCtx T;
             T.keys = (uint64_t *)(tbase + TB.off_keys);
             T.c32 = (uint32_t *)(tbase + TB.off_cnts);
+            T.list = (uint16_t *)(tbase + TB.off_list);
             T.cap = TB.cap;
             T.rseq = gR;   // REF keys store read indices relative to gR
             T.SW = SW;
@@ -1465,6 +1432,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
             TabCtx T;
             T.keys = (uint64_t *)(sm + TB.off_keys);
             T.c32 = (uint32_t *)(sm + TB.off_cnts);
+            T.list = (uint16_t *)(sm + TB.off_list);
             T.cap = TB.cap;
             T.rseq = sR;
             T.SW = SW;
