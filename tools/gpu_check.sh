@@ -1,5 +1,5 @@
 #!/bin/bash
-# One GPU verification pass: build, GPU parity tests, smoke, bench line, ncu launch list.
+# One GPU verification pass: build, GPU parity tests, smoke, bench line, ncu launch list, one full capture.
 set -x
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/gpu.txt 2>&1
@@ -8,4 +8,7 @@ timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
 timeout 1200 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.json 2> gpurun_out/bench.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > gpurun_out/ncu_bench.log 2>&1
+if [ -n "$FULL" ]; then
+  timeout 1200 ncu --set full --import-source on --clock-control none -k regex:"$FULL" --launch-count 1 -o gpurun_out/top_full python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e > gpurun_out/ncu_full.log 2>&1
+fi
 echo done
