@@ -913,16 +913,18 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
         }
         t_filter = clock64();
         // ---- build (Alg 1) ----
-        warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
-                       [&](bool act, const PosV &v) {
-                           const uint64_t h = hash_kmer(v.K, KW);
-                           bool want = act;
-                           if (mbits) {
-                               const uint32_t fi = filt_index(h, mbits);
-                               want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
-                           }
-                           warp_insert<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
-                       });
+        {
+            warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                      [&](bool act, const PosV &v) {
+                          const uint64_t h = hash_kmer(v.K, KW);
+                          bool want = act;
+                          if (mbits) {
+                              const uint32_t fi = filt_index(h, mbits);
+                              want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+                          }
+                          warp_insert<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
+                      });
+        }
     } else {
         constexpr int NW = MAX_KW;
         // ---- filter pass (REF keys, k >= 64: rare; per-thread rolling traversal) ----

@@ -419,7 +419,7 @@ extern "C" la_status la_load_batch(la_ctx *ctx, const la_batch *b, const la_para
             CK(cudaMemsetAsync(E.rflag.p, 0, nR, st));
             k_read_end<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(E.eoff), nE, nR, P<int32_t>(ctx->read_end));
             CKL();
-            k_encode_reads<<<blocks(nR * SW, 256), 256, 0, st>>>(
+            k_encode_reads_staged<<<blocks(nR, ENC_R), 256, 0, st>>>(
                 d_seq, d_qual, P<int64_t>(E.roff), P<int32_t>(ctx->read_end), nR, SW, dp, P<uint64_t>(E.rseq),
                 P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), d_err);
             CKL();
