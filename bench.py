@@ -224,6 +224,9 @@ def run_reference(args):
     if rank != 0:
         return 0
     batch, params = load_workload(args.config, 0, args.scale)
+    if args.k_start:
+        params = params.replace(k_start=args.k_start, k_min=min(params.k_min, args.k_start),
+                                k_max=max(params.k_max, args.k_start))
     vals = []
     for step in range(args.warmup + args.steps):
         v, eps, cores, desc = cpu_oracle_sample(batch, params, budget_s=args.ref_budget, seed=step)
@@ -234,7 +237,8 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": CONFIG_DESC[args.config], "n_ends": batch.n_ends, "n_reads": batch.n_reads},
+            "config": {"workload": CONFIG_DESC[args.config] + (f", k_start={args.k_start}" if args.k_start else ""),
+                       "n_ends": batch.n_ends, "n_reads": batch.n_reads},
             "contig_ends_per_s": eps,
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
                              "sample": vals[-1][2]},
@@ -255,6 +259,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-chunks", type=int, default=8)
+    ap.add_argument("--k-start", type=int, default=None,
+                    help="NEXT N2: LA at another k of the assembler's contig iteration (21, 33, 55, 77)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -268,6 +274,9 @@ def main():
     barrier(world)
     torch.cuda.set_device(local)
     batch, params = load_workload(args.config, rank, args.scale)
+    if args.k_start:
+        params = params.replace(k_start=args.k_start, k_min=min(params.k_min, args.k_start),
+                                k_max=max(params.k_max, args.k_start))
     stream = torch.cuda.Stream()
     la = LocalAssembler(local, stream=stream)
 
@@ -368,7 +377,9 @@ def main():
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": CONFIG_DESC[args.config], "n_ends": batch.n_ends, "n_contigs": batch.n_contigs,
+        "config": {"workload": CONFIG_DESC[args.config] + (f", k_start={args.k_start}" if args.k_start else ""),
+                   "k_schedule": [params.k_start, params.k_min, params.k_max, params.k_shift],
+                   "n_ends": batch.n_ends, "n_contigs": batch.n_contigs,
                    "n_reads": batch.n_reads, "scale": args.scale, "seed": "20211114+cfg+rank",
                    "l2": "flushed between timed steps (256 MB write)", "parallelism": f"contig-shards x{world}"},
         "contig_ends_per_s": ends_per_s,

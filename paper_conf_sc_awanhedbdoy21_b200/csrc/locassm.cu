@@ -64,6 +64,7 @@ struct la_ctx {
     int cls_threads[N_SMEM_CLASSES] = {64, 128, 256, 256, 512};
     int cls_ctas[N_SMEM_CLASSES] = {12, 6, 3, 2, 1};   // resident CTAs per SM of each shared-memory class
     uint32_t cls_bytes[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};   // dynamic shared memory per CTA
+    uint32_t xl_bytes = 0;        // dynamic shared memory of the XL class (the rest of the SM's 228 KB is L1)
     uint32_t small_mask = 0x3u;   // classes run by k_small (one end per CTA, no walker warp)
     la_params params{};
     DevParams dp{};
@@ -207,6 +208,13 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - 512);
         ctx->cls_bytes[i] = (uint32_t)(per & ~(size_t)127);
     }
+    // XL: tables live in L2; shared memory holds the link words and filter bitmaps, and whatever the
+    // class leaves unused becomes L1 for the end's streamed reads (tuning hook LA_XL_SMEM_KB)
+    ctx->xl_bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
+    if (const char *x = getenv("LA_XL_SMEM_KB")) {
+        const uint32_t b = (uint32_t)atoi(x) * 1024u;
+        if (b >= 96u * 1024u && b < ctx->xl_bytes) ctx->xl_bytes = b;
+    }
     if (cuda_stream) ctx->stream = (cudaStream_t)cuda_stream;
     else {
         if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess) {
@@ -227,6 +235,11 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     if (getenv("LA_SERIAL_CLASSES") && atoi(getenv("LA_SERIAL_CLASSES"))) ctx->concurrent_classes = false;
     bool attr_ok = cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         ctx->cls_bytes[N_SMEM_CLASSES - 1]) == cudaSuccess;
+    {   // XL: ask for the smallest shared-memory carveout that holds xl_bytes (the rest is L1)
+        const int pct = (int)std::min<size_t>(100, ((size_t)ctx->xl_bytes + 2048) * 100 / prop.sharedMemPerMultiprocessor + 1);
+        attr_ok &= cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                        pct) == cudaSuccess;
+    }
     {
         uint32_t mx = 0;
         for (int i = 0; i < N_SMEM_CLASSES; ++i) mx = std::max(mx, ctx->cls_bytes[i]);
@@ -601,7 +614,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         if (force_smem) pb.b[0] = 0xffffffffu;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
             P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
-            (force_global || force_smem) ? 0u : ctx->cls_bytes[N_SMEM_CLASSES - 1], P<int32_t>(ctx->cls),
+            (force_global || force_smem) ? 0u : ctx->xl_bytes, P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
             lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
@@ -650,7 +663,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(cudaEventRecord(ctx->ev_cls0[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));
     if (n_xl > 0) {
         cudaStream_t st = cls_st(N_SMEM_CLASSES);
-        const uint32_t bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
+        const uint32_t bytes = ctx->xl_bytes;
         const uint32_t icap = smem_fixed(dp.W, bytes, 1u).icap;
         const uint32_t stride = xl_stride(xl_rmax, xl_umax, dp.V >= 2, icap);
         const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm, n_xl);

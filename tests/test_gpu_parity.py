@@ -240,3 +240,11 @@ def test_streamed_edge_cases(LA, orc):
         setattr(d, f, torch.from_numpy(getattr(small, f)).cuda())
     with pytest.raises(LocAssmError, match="host batch"):
         LA.extend_streamed(d, P0, 2)
+
+
+@pytest.mark.parametrize("k_start", [21, 55, 77])
+def test_assembler_k_rounds(LA, orc, k_start):
+    """NEXT N2: local assembly at the other k of the assembler's contig iteration (Fig 1 "iterate
+    for k", P:L150-160); k_start 77 starts on pointer (REF) keys, 55 upshifts into them."""
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(400))
+    check(LA, orc, b, P0.replace(k_start=k_start, k_min=21, k_max=99))
