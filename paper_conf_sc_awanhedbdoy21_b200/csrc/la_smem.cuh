@@ -587,11 +587,12 @@ __device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, con
     const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
     const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
     if (wb >= we) return;
+    uint64_t m0, m1;
+    kmer_masks(k, m0, m1);
     constexpr uint32_t SPAN = 32u * RUN;
-    uint32_t g = wb + (uint32_t)lane * RUN;
     int j;
     {   // read j with pref[j] <= g < pref[j+1]
-        const uint32_t gg = min(g, we - 1);
+        const uint32_t gg = min(wb + (uint32_t)lane * RUN, we - 1);
         int lo = 0, hi = r;
         while (hi - lo > 1) {
             const int mid = (lo + hi) >> 1;
@@ -599,36 +600,42 @@ __device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, con
         }
         j = lo;
     }
-    for (uint32_t base = wb; base < we; base += SPAN, g += SPAN) {
-        if (__shfl_sync(0xffffffffu, *stop, 0)) return;
-        KmerN<2> K;
-        K.w[0] = K.w[1] = 0;
-        int p = 0, lastN = -1, npos = 0;
-        const uint64_t *R = rseq, *Q = rqc;
-        bool flag = false;
-        // (re)start: extract the k-mer at position g (read j) — at the run start and at a read change
-        auto start = [&](uint32_t gpos) {
-            uint32_t pj = pref[j + 1];
-            while (pj <= gpos) pj = pref[++j + 1];   // skips reads without positions
-            const uint32_t pj0 = pref[j];
-            p = (int)(gpos - pj0);
-            npos = (int)(pj - pj0);
-            const long long rid = r0 + j;
-            R = rseq + rid * SW;
-            Q = rqc + rid * SW;
-            flag = rflag[rid] != 0;
-            K = extract_kmer<2>(R, p, k, KW);
-            lastN = -1;
-            if (flag)
-                for (int i = p; i < p + k; ++i)
-                    if (get2(Q, i) == 3u) lastN = i;
-        };
-        if (g < we) start(g);
-#pragma unroll
-        for (int i = 0; i < RUN; ++i) {
-            const uint32_t gi = g + (uint32_t)i;
-            const bool act = gi < we;
-            if (act && i > 0 && p >= npos) start(gi);   // the run crossed into the next read
+    uint32_t pj0 = pref[j], pj1 = pref[j + 1];
+    const uint64_t *R = rseq + (r0 + j) * SW, *Q = rqc + (r0 + j) * SW;
+    bool flag = rflag[r0 + j] != 0;
+    KmerN<2> K;
+    K.w[0] = K.w[1] = 0;
+    int p = 0, lastN = -1;
+    uint32_t g = wb + (uint32_t)lane * RUN;   // this lane's next position
+    for (uint32_t base = wb; base < we; base += SPAN) {
+        if (((base - wb) & (4u * SPAN - 1u)) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;
+        g = base + (uint32_t)lane * RUN;
+#pragma unroll 1
+        for (int i = 0; i < RUN; ++i, ++g) {
+            const bool act = g < we;
+            if (act && (i == 0 || g >= pj1)) {   // (re)start: run start or the run entered a later read
+                if (g >= pj1) {
+                    do {
+                        pj0 = pj1;
+                        pj1 = pref[++j + 1];
+                    } while (g >= pj1);
+                    R = rseq + (r0 + j) * SW;
+                    Q = rqc + (r0 + j) * SW;
+                    flag = rflag[r0 + j] != 0;
+                }
+                p = (int)(g - pj0);
+                const int q = p >> 5, sft = (p & 31) << 1, q2 = min(q + 2, SW - 1);
+                const uint64_t w0 = R[q], w1 = R[q + 1], w2 = R[q2];
+                K.w[0] = funnel64(w0, w1, sft) & m0;
+                K.w[1] = funnel64(w1, w2, sft) & m1;
+                lastN = -1;
+                if (flag) {   // last N inside the window [p, p+k) (bit 62-2i of nmask marks base i)
+                    const uint64_t n0 = nmask_word(Q[q]), n1 = nmask_word(Q[q + 1]), n2 = nmask_word(Q[q2]);
+                    const uint64_t N0 = funnel64(n0, n1, sft) & m0, N1 = funnel64(n1, n2, sft) & m1;
+                    lastN = N1 ? p + 32 + ((62 - (__ffsll((long long)N1) - 1)) >> 1)
+                               : (N0 ? p + ((62 - (__ffsll((long long)N0) - 1)) >> 1) : -1);
+                }
+            }
             PosV v;
             v.vote = false;
             v.nb = 0;
@@ -643,7 +650,7 @@ __device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, con
             }
             v.K = K;
             f(act && v.vote, v);
-            if (i + 1 < RUN && act) {
+            if (act) {   // next_kmer (Alg 2 line 15) for the lane's next position
                 roll_kmer(K, k, KW, v.nb);
                 ++p;
             }
