@@ -365,11 +365,20 @@ def main():
         return 0
     peaks = roofline_peaks()
     roof = None
+    hbm_bytes_alg = int(batch.read_seq.nbytes) // 4 * 2   # packed reads (2-bit seq + 2-bit qual) streamed once per step
     if peaks["smem_gups"]:
         ach = st["inserts_smem"] / (ms_smem / 1e3) / 1e9 if ms_smem > 0 else 0.0
-        roof = {"bound": "smem", "kernel": "k_smem (shared-memory table build+walk)",
+        traffic, tsrc = None, None
+        try:   # DRAM bytes per step of the table kernels from the committed ncu capture (tools/traffic.py)
+            tj = json.load(open(os.path.join(ROOT, "profiles", "r01_traffic.json")))
+            traffic = tj["table_kernels_per_step"]["dram_bytes"]
+            tsrc = "profiles/r01_traffic.json (ncu dram__bytes_read.sum + dram__bytes_write.sum, table kernels, per step)"
+        except Exception:
+            pass
+        roof = {"bound": "smem", "kernel": "k_small / k_smem (table build + link + walk, all classes)",
                 "achieved": ach, "peak": peaks["smem_gups"], "unit": "G updates/s",
-                "frac": ach / peaks["smem_gups"], "traffic": None,
+                "frac": ach / peaks["smem_gups"], "traffic": traffic, "traffic_src": tsrc,
+                "algorithmic_bytes": hbm_bytes_alg,
                 "peak_src": peaks["smem_src"],
                 "note": "algorithmic unit = one vote insert (1 random table update); see DESIGN.md §7"}
     hbm_bytes = int(batch.read_seq.nbytes) // 4 * 2   # packed reads (2-bit seq + 2-bit qual) streamed once per step

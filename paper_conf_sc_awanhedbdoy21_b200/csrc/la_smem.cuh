@@ -1,26 +1,26 @@
-// la_smem.cuh — planner and the shared-memory-table kernel.
+// la_smem.cuh — planner and the table kernels.
 //
-// k_smem: persistent CTAs; each CTA = one walker warp + (BLOCK-32) builder threads and keeps TWO
-// contig ends in flight, so the serial mer-walk of one end overlaps the table build of the other.
-//   builders, per attempt (k) of an end:
-//     [filter pass]  only when the unfiltered table may not fit: every voting k-mer occurrence sets a
-//                    bit in B1 (atomicOr); a second sighting sets its bit in B2.  k-mers with fewer
-//                    than two voting occurrences cannot reach min_votes >= 2, so they extend exactly
-//                    like absent k-mers (DEADEND) and may be left out (reading #4); bitmap collisions
-//                    only admit extra k-mers, never exclude one.
-//     [build, Alg 1] every voting occurrence of a k-mer that passed the filter is
-//                    inserted into an open-addressing table in shared memory.  k <= 63: the slot holds
-//                    the 2-bit k-mer itself (16 B) and is claimed with one 128-bit CAS; k >= 64: the slot
-//                    holds tag|read|pos (pointer-encoded key) verified against the read.
-//                    The vote for the following base goes to packed 8-bit counters lo[4],
-//                    hi[4] (32-bit atomicAdds; an 8-bit carry is detected -> redo in the global path).
-//     [link]         per slot: ext(lo, hi) (reading #1) and, for a base, the slot of the successor
-//                    k-mer (next_kmer, Alg 2 line 15) -> an info word in the end's own info buffer.
-//   walker (lane 0 of warp 0): follows the info words from the start k-mer (Alg 2) with a
-//     visited bit per slot (the loop-check table), then applies the k-shift rule
-//      and hands the end back to the builders (next k) or writes its result.
-// Reads are not staged: builders stream them from HBM/L2 (up to 2 passes per attempt).  Table
-// overflow (claims above 70% of capacity) or a counter carry re-routes the end to the global path.
+// Per attempt (one k) of one contig end, `build_link` runs on the CTA's builder warps:
+//   [filter pass]  only when the unfiltered table may not fit: every voting k-mer occurrence sets a
+//                  bit in B1 (atomicOr); a second sighting sets its bit in B2.  k-mers with fewer than
+//                  two voting occurrences cannot reach min_votes >= 2, so they extend exactly like
+//                  absent k-mers (DEADEND) and may be left out (reading #4); bitmap collisions only
+//                  admit extra k-mers, never exclude one.
+//   [build, Alg 1] every voting occurrence that passed the filter is inserted into an
+//                  open-addressing table (shared memory; XL: L2-resident global scratch).  k <= 63: the
+//                  slot holds the 2-bit k-mer itself (16 B), claimed with one 128-bit CAS; k >= 64: the
+//                  slot holds tag|read|pos (pointer key), verified against the read.  The
+//                  vote for the following base is one atomic on 8-bit counters (high-tier
+//                  and low-only words; a carry re-routes the end to the global path).
+//   [link]         per claimed slot (claim list): ext(lo, hi) (reading #1) and, for a base, the slot of
+//                  the successor k-mer (next_kmer, Alg 2 line 15) -> a link word.
+// All three passes are warp-convergent: lane per position (or per claimed slot), whole-warp probe
+// rounds, claims counted once per warp.
+// The walk (Alg 2) follows the link words from the start k-mer with a visited bit per
+// slot (the loop-check table), then the k-shift rule picks the next k.
+//   k_small (small tables): one end per CTA; every warp builds, thread 0 walks; reads staged once.
+//   k_smem  (larger tables): one walker warp + builders, two ends in flight (mbarrier hand-off), so
+//           the walk of one end overlaps the build of the other; XL streams reads from L2/HBM.
 #pragma once
 #include "la_device.cuh"
 
@@ -362,115 +362,6 @@ __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> 
     return NONE;
 }
 
-// Alg 1 line 5 (kmer_ht.insert) with the vote of the following base.
-template <bool INL, bool GT, int NW>
-__device__ __forceinline__ void tab_insert(const TabCtx &T, const KmerN<NW> &K, uint64_t h, uint32_t rid, int pos,
-                                           uint32_t b, bool hi, int *nclaim, int claim_limit, volatile int *ovf) {
-    uint32_t s = slot_of(h, T.cap);
-    if (INL) {
-        uint64_t a, bb;
-        inline_form(K, T.KW, a, bb);
-        for (;;) {
-            uint64_t x, y;
-            ld128v<GT>(&T.keys[2 * s], x, y);
-            if (y == 0) {   // looks empty: the CAS either claims it or returns its true content
-                if (*ovf) return;
-                cas128<GT>((void *)&T.keys[2 * s], 0ull, 0ull, a, bb, x, y);
-                if (y == 0) {   // claimed
-                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
-                    break;
-                }
-            } else if (y == bb && x != a) {
-                // a 16 B load is not guaranteed single-copy atomic: if it raced with the claiming CAS,
-                // word 0 may be stale — re-read it (a slot never changes once claimed)
-                x = *(volatile uint64_t *)&T.keys[2 * s];
-            }
-            if (x == a && y == bb) break;
-            s = (s + 1 == T.cap) ? 0 : s + 1;
-        }
-    } else {
-        const uint64_t tag = tag_of(h);
-        volatile uint64_t *vk = T.keys;
-        for (;;) {
-            uint64_t w = vk[s];
-            if (w == 0) {
-                if (*ovf) return;
-                const uint64_t mine = make_slot(tag, rid, (uint32_t)pos);
-                const uint64_t old = atomicCAS((unsigned long long *)&T.keys[s], 0ull, (unsigned long long)mine);
-                if (old == 0) {
-                    if (atomicAdd(nclaim, 1) >= claim_limit) *ovf = 1;
-                    break;
-                }
-                w = old;
-            }
-            if ((w & TAG_MASK) == tag) {
-                const KmerN<NW> K2 = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
-                if (kmer_eq(K, K2, T.KW)) break;
-            }
-            s = (s + 1 == T.cap) ? 0 : s + 1;
-        }
-    }
-    vote_add<GT>(T, s, b, hi, ovf);
-}
-
-// Every voting occurrence of the end's reads (staged in shared memory, or streamed from global memory
-// for the XL class: plain generic loads serve both).  The end's positions with a
-// following base are numbered 0..total-1 read by read (pref[j] = first number of read j); builder bt
-// takes the contiguous range [bt*total/NB, (bt+1)*total/NB), so work is balanced to one position and a
-// thread extracts a k-mer only where its range enters a read, then rolls it; the following base and
-// its quality class come from one 64-bit word per 32 positions.  f(K, rid, p, nb, hi) per vote.
-template <int NW, typename F>
-__device__ __forceinline__ void for_each_vote(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
-                                              const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
-                                              const uint32_t *pref, int64_t r0, int r, int SW, int k, int KW,
-                                              int bt, int NB, const volatile int *stop, F &&f) {
-    const uint32_t total = pref[r];
-    uint32_t cur = (uint32_t)(((uint64_t)total * (uint32_t)bt) / (uint32_t)NB);
-    const uint32_t end = (uint32_t)(((uint64_t)total * (uint32_t)(bt + 1)) / (uint32_t)NB);
-    if (cur >= end) return;
-    int lo = 0, hi = r;   // read j with pref[j] <= cur < pref[j+1]
-    while (hi - lo > 1) {
-        const int mid = (lo + hi) >> 1;
-        if (pref[mid] <= cur) lo = mid; else hi = mid;
-    }
-    int j = lo;
-    while (pref[j + 1] <= cur) ++j;   // skip reads without positions
-    int p = (int)(cur - pref[j]);
-    while (cur < end) {
-        if (*stop) return;
-        const int64_t rid = r0 + j;
-        const int npos = (int)(pref[j + 1] - pref[j]);   // = len - k > 0
-        const int pe = min(npos, p + (int)(end - cur));
-        const uint64_t *R = rseq + rid * SW;
-        const uint64_t *Q = rqc + rid * SW;
-        KmerN<NW> K = extract_kmer<NW>(R, p, k, KW);
-        int lastN = -1;
-        if (rflag[rid])   // this read has an N
-            for (int i = p; i < p + k; ++i)
-                if (get2(Q, i) == 3u) lastN = i;
-        int wi = (p + k) >> 5;
-        uint64_t wR = R[wi], wQ = Q[wi];
-        for (int q = p; q < pe; ++q) {
-            const int i = q + k;
-            if ((i >> 5) != wi) {
-                wi = i >> 5;
-                wR = R[wi];
-                wQ = Q[wi];
-            }
-            const int sh = 62 - ((i & 31) << 1);
-            const uint32_t nb = (uint32_t)(wR >> sh) & 3u;
-            const uint32_t nq = (uint32_t)(wQ >> sh) & 3u;
-            if (nq - 1u < 2u && lastN < q) f(K, (uint32_t)rid, q, nb, nq == 2u);
-            if (nq == 3u) lastN = i;
-            roll_kmer(K, k, KW, nb);
-        }
-        cur += (uint32_t)(pe - p);
-        ++j;
-        p = 0;
-        while (cur < end && pref[j + 1] == pref[j]) ++j;
-    }
-}
-
 #ifdef LA_PROBE_STATS
 // debug build only: [0] warp_insert calls, [1] probe rounds, [2] inserting lanes, [3] claims,
 // [4] lookup calls, [5] lookup rounds, [6] looking-up lanes, [7] sum of table loads at link (claims*1000/cap)
@@ -738,6 +629,158 @@ __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const Po
     if (found) vote_add<GT>(T, hit, v.nb, v.hi, ovf);
 }
 
+// ---- warp-convergent passes for pointer keys (k >= 64) ----------------------------------------
+struct PosR {            // one lane's position, k-mer of up to 4 words
+    KmerN<MAX_KW> K;
+    uint32_t nb, rid;    // following base, read index (relative to the key rows)
+    int p;
+    bool vote, hi;
+};
+
+// f(act, v) per warp iteration, lane-per-position as warp_positions, for k <= 128.
+template <typename F>
+__device__ __forceinline__ void warp_positions_ref(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
+                                                   const uint8_t *__restrict__ rflag, const uint32_t *pref,
+                                                   long long r0, int r, int SW, int k, int KW, int wid, int nwarps,
+                                                   int lane, const volatile int *stop, F &&f) {
+    const uint32_t total = pref[r];
+    const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
+    const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
+    if (wb >= we) return;
+    uint32_t g = wb + lane;
+    int j;
+    {
+        const uint32_t gg = min(g, we - 1);
+        int lo = 0, hi = r;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (pref[mid] <= gg) lo = mid; else hi = mid;
+        }
+        j = lo;
+    }
+    uint32_t pj0 = pref[j], pj1 = pref[j + 1];
+    for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
+        if (((base - wb) & 127u) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;
+        const bool act = g < we;
+        PosR v;
+        v.vote = false;
+        v.nb = 0;
+        v.hi = false;
+        v.p = 0;
+        v.rid = 0;
+#pragma unroll
+        for (int w = 0; w < MAX_KW; ++w) v.K.w[w] = 0;
+        if (act) {
+            while (g >= pj1) {
+                pj0 = pj1;
+                pj1 = pref[++j + 1];
+            }
+            const long long rid = r0 + j;
+            const uint64_t *R = rseq + rid * SW, *Q = rqc + rid * SW;
+            const int p = (int)(g - pj0);
+            v.K = extract_kmer<MAX_KW>(R, p, k, KW);
+            v.p = p;
+            v.rid = (uint32_t)rid;
+            const int i = p + k, sh = 62 - ((i & 31) << 1);
+            v.nb = (uint32_t)(R[i >> 5] >> sh) & 3u;
+            const uint32_t nq = (uint32_t)(Q[i >> 5] >> sh) & 3u;
+            v.vote = nq - 1u < 2u;
+            v.hi = nq == 2u;
+            if (v.vote && rflag[rid]) {   // reading #5: any N in [p, p+k) -> no entry
+                const int q = p >> 5, s2 = (p & 31) << 1;
+#pragma unroll
+                for (int w = 0; w < MAX_KW; ++w) {
+                    const int bits = 2 * k - 64 * w;
+                    const uint64_t m = bits >= 64 ? ~0ull : (bits > 0 ? (~0ull << (64 - bits)) : 0ull);
+                    const uint64_t n = funnel64(nmask_word(Q[q + w]), nmask_word(Q[q + w + 1]), s2) & m;
+                    if (w < KW && n) v.vote = false;
+                }
+            }
+        }
+        f(act && v.vote, v);
+    }
+}
+
+// Convergent insert with pointer keys: a round probes one slot; a tag match is verified against the
+// k-mer at the slot's (read, pos) in the staged reads (exact equality).
+template <bool GT>
+__device__ __forceinline__ uint32_t ref_probe_find(const TabCtx &T, const KmerN<MAX_KW> &K, uint64_t tag, uint64_t w) {
+    if ((w & TAG_MASK) != tag) return 0u;
+    const KmerN<MAX_KW> K2 = extract_kmer<MAX_KW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
+    return kmer_eq(K, K2, T.KW) ? 1u : 0u;
+}
+
+template <bool GT>
+__device__ __forceinline__ void warp_insert_ref(const TabCtx &T, bool want, const PosR &v, uint64_t h, int lane,
+                                                int *nclaim, int claim_limit, volatile int *ovf) {
+    uint32_t s = slot_of(h, T.cap), hit = 0;
+    const uint64_t tag = tag_of(h), mine = make_slot(tag, v.rid, (uint32_t)v.p);
+    bool pend = want, found = false;
+    volatile uint64_t *vk = T.keys;
+    while (__any_sync(0xffffffffu, pend)) {
+        bool claimed = false;
+        if (pend) {
+            uint64_t w = vk[s];
+            if (w == 0) {
+                if (*ovf) {
+                    pend = false;
+                } else {
+                    w = atomicCAS((unsigned long long *)&T.keys[s], 0ull, (unsigned long long)mine);
+                    if (w == 0) {
+                        claimed = true;
+                        pend = false;
+                        found = true;
+                        hit = s;
+                    }
+                }
+            }
+            if (pend && w != 0) {
+                if (ref_probe_find<GT>(T, v.K, tag, w)) {
+                    pend = false;
+                    found = true;
+                    hit = s;
+                } else {
+                    s = (s + 1 == T.cap) ? 0 : s + 1;
+                }
+            }
+        }
+        const unsigned cm = __ballot_sync(0xffffffffu, claimed);
+        if (cm) {
+            const int n = __popc(cm), leader = __ffs(cm) - 1;
+            int first = 0;
+            if (lane == leader) {
+                first = atomicAdd(nclaim, n);
+                if (first + n > claim_limit) *ovf = 1;
+            }
+            first = __shfl_sync(0xffffffffu, first, leader);
+            if (claimed) T.list[first + __popc(cm & ((1u << lane) - 1u))] = (uint16_t)hit;
+        }
+    }
+    if (found) vote_add<GT>(T, hit, v.nb, v.hi, ovf);
+}
+
+template <bool GT>
+__device__ __forceinline__ uint32_t warp_lookup_ref(const TabCtx &T, bool want, const KmerN<MAX_KW> &K, uint64_t h) {
+    uint32_t s = slot_of(h, T.cap), res = NONE, n = 0;
+    const uint64_t tag = tag_of(h);
+    bool pend = want;
+    while (__any_sync(0xffffffffu, pend)) {
+        if (pend) {
+            const uint64_t w = T.keys[s];
+            if (w == 0) {
+                pend = false;
+            } else if (ref_probe_find<GT>(T, K, tag, w)) {
+                pend = false;
+                res = s;
+            } else {
+                s = (s + 1 == T.cap) ? 0 : s + 1;
+                if (++n >= T.cap) pend = false;
+            }
+        }
+    }
+    return res;
+}
+
 // Convergent lookup (no insert): slot of K or NONE; slot pairs as in warp_insert.
 template <bool GT>
 __device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, const KmerN<2> &K, uint64_t h) {
@@ -933,30 +976,31 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                       });
         }
     } else {
-        constexpr int NW = MAX_KW;
-        // ---- filter pass (REF keys, k >= 64: rare; per-thread rolling traversal) ----
+        // ---- pointer keys (k >= 64): the same passes with 4-word k-mers ----
         if (mbits) {
-            for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                              [&](const KmerN<NW> K, uint32_t, int, uint32_t, bool) {
-                                  const uint32_t fi = filt_index(hash_kmer(K, KW), mbits);
-                                  const uint32_t bit = 1u << (fi & 31);
-                                  if (!(B2[fi >> 5] & bit)) {
-                                      const uint32_t old = atomicOr(&B1[fi >> 5], bit);
-                                      if (old & bit) atomicOr(&B2[fi >> 5], bit);
-                                  }
-                              });
+            warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                               [&](bool act, const PosR &v) {
+                                   if (!act) return;
+                                   const uint32_t fi = filt_index(hash_kmer(v.K, KW), mbits);
+                                   const uint32_t bit = 1u << (fi & 31);
+                                   if (!(*(volatile uint32_t *)&B2[fi >> 5] & bit)) {
+                                       const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                       if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                                   }
+                               });
             builders_sync(NB);
         }
         t_filter = clock64();
-        for_each_vote<NW>(T.rseq, rqc, rlen, rflag, pref, r0, r, T.SW, k, KW, bt, NB, stop,
-                          [&](const KmerN<NW> K, uint32_t rid, int p, uint32_t nb, bool hi) {
-                              const uint64_t h = hash_kmer(K, KW);
-                              if (mbits) {
-                                  const uint32_t fi = filt_index(h, mbits);
-                                  if (!((B2[fi >> 5] >> (fi & 31)) & 1u)) return;
-                              }
-                              tab_insert<false, GT, NW>(T, K, h, rid, p, nb, hi, &B.nclaim, claim_limit, &B.overflow);
-                          });
+        warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                           [&](bool act, const PosR &v) {
+                               const uint64_t h = hash_kmer(v.K, KW);
+                               bool want = act;
+                               if (mbits) {
+                                   const uint32_t fi = filt_index(h, mbits);
+                                   want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+                               }
+                               warp_insert_ref<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
+                           });
     }
     builders_sync(NB);
     t_build = clock64();
@@ -991,20 +1035,25 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             link_batch(i < nocc, i < nocc ? (uint32_t)T.list[i] : 0u);
         }
     } else {
-        constexpr int NW = MAX_KW;
-        for (uint32_t s = bt; s < T.cap; s += NB) {
-            const uint64_t w = T.keys[s];
-            if (w == 0) continue;
-            KmerN<NW> K = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
-            uint32_t lo[4], hi[4];
-            votes_of<GT>(T, s, lo, hi);
-            const int code = ext_rule(lo, hi, P.V, P.F);
-            uint32_t nxt = NONE;
-            if (code < 4) {
-                roll_kmer(K, k, KW, (uint32_t)code);
-                nxt = tab_lookup<false, NW>(T, K, hash_kmer(K, KW));
+        const uint32_t nocc = min((uint32_t)B.nclaim, T.cap);
+        for (uint32_t base = (uint32_t)wid * 32u; base < nocc; base += (uint32_t)NB) {
+            const uint32_t i = base + lane;
+            const bool has = i < nocc;
+            const uint32_t s = has ? (uint32_t)T.list[i] : 0u;
+            KmerN<MAX_KW> K;
+#pragma unroll
+            for (int w = 0; w < MAX_KW; ++w) K.w[w] = 0;
+            int code = CODE_DEADEND;
+            if (has) {
+                const uint64_t w = T.keys[s];
+                K = extract_kmer<MAX_KW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
+                uint32_t lo[4], hi[4];
+                votes_of<GT>(T, s, lo, hi);
+                code = ext_rule(lo, hi, P.V, P.F);
+                if (code < 4) roll_kmer(K, k, KW, (uint32_t)code);
             }
-            info[s] = link_info(code, nxt);
+            const uint32_t t = warp_lookup_ref<GT>(T, has && code < 4, K, hash_kmer(K, KW));
+            if (has) info[s] = link_info(code, t);
         }
     }
     if (bt == 0) {
