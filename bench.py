@@ -132,6 +132,7 @@ def roofline_peaks():
     try:
         m = json.load(open(os.path.join(ROOT, "profiles", "micro_random_update.json")))
         peaks["smem_gups"] = m["smem_atomic_add32"]
+        peaks["insert_gups"] = m.get("smem_hash_insert")
         peaks["smem_src"] = "profiles/micro_random_update.json (smem_atomic_add32, measured on B200)"
     except Exception:
         peaks["smem_gups"] = None
@@ -407,6 +408,12 @@ def main():
                              for i, n in enumerate(["smem64x12", "smem128x6", "smem256x3", "smem256x2",
                                                     "smem512x1", "xl512x1"])}},
         "roofline": roof,
+        "roofline_insert": ({"bound": "smem", "kernel": roof["kernel"], "achieved": roof["achieved"],
+                             "peak": peaks["insert_gups"], "unit": "G inserts/s",
+                             "frac": roof["achieved"] / peaks["insert_gups"],
+                             "peak_src": "profiles/micro_random_update.json smem_hash_insert: the table's insert "
+                                         "primitive alone (hash + slot-pair probe + vote atomic), measured on B200"}
+                            if roof and peaks.get("insert_gups") else None),
         "roofline_hbm": {"bound": "hbm", "achieved": hbm_bytes / (ms_max / args.steps / 1e3) / 1e9,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": hbm_bytes / (ms_max / args.steps / 1e3) / 1e9 / peaks["hbm_gbs"],
