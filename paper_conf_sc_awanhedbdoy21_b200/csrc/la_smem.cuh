@@ -1282,7 +1282,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         const uint64_t *gQ = GT ? rqc : sQ;
         const uint16_t *gL = GT ? rlen : sL;
         const uint8_t *gF = GT ? rflag : sF;
-        const long long lr0 = GT ? r0 : 0;   // first read index in (gR, gQ, gL, gF)
+        long long lr0 = GT ? r0 : 0;   // first read index in (gR, gQ, gL, gF)
         if (!GT && !no_room) {
             const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
             const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
@@ -1307,7 +1307,39 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         const long long tc = clock64();
         b_t[1] += tc - tb;
         long long td = tc, t_filter = tc, t_build = tc;
-        SmemTab TB = smem_tab(FX, U, P.V >= 2, key_bytes(k), r, GT, SW);
+        // XL: stage this end's reads in shared memory when they fit beside the filter bitmaps (the
+        // streamed reads were the XL kernel's top stall: long scoreboard on L2, ncu r01)
+        SmemFixed FXt = FX;
+        if (GT && !no_room) {
+            const uint32_t xs = (stage_bytes(r, SW) + 127u) & ~127u;
+            const uint32_t mw = ((4u * U + 31u) / 32u + 3u) & ~3u;
+            if (xs + 8u * mw + 256u <= FX.filt_bytes) {
+                uint64_t *xR = (uint64_t *)(sm + FX.off_filt);
+                uint64_t *xQ = xR + (size_t)r * SW;
+                uint16_t *xL = (uint16_t *)(xQ + (size_t)r * SW);
+                uint8_t *xF = (uint8_t *)(xL + r);
+                const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
+                const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
+                const int n4 = r * SW / 2;   // SW is even
+                for (int i = bt; i < n4; i += NB) {
+                    ((uint4 *)xR)[i] = __ldg(&a4[i]);
+                    ((uint4 *)xQ)[i] = __ldg(&b4[i]);
+                }
+                for (int i = bt; i < r; i += NB) {
+                    xL[i] = __ldg(&rlen[r0 + i]);
+                    xF[i] = __ldg(&rflag[r0 + i]);
+                }
+                builders_sync(NB);
+                gR = xR;
+                gQ = xQ;
+                gL = xL;
+                gF = xF;
+                lr0 = 0;
+                FXt.off_filt += xs;
+                FXt.filt_bytes -= xs;
+            }
+        }
+        SmemTab TB = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW);
         if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
             const uint32_t need = xl_needed_cap(r, U, TB.mwords != 0);
             if (TB.cap > need) {
