@@ -27,7 +27,10 @@
 namespace la {
 
 enum : int { CLS_NOREADS = 0, CLS_SHORT = 1, CLS_S = 2, CLS_GLOBAL = 8 };   // CLS_S + class index (5 = XL)
-constexpr float SMEM_MAX_LOAD = 0.70f;
+#ifndef LA_MAX_LOAD
+#define LA_MAX_LOAD 0.70f
+#endif
+constexpr float SMEM_MAX_LOAD = LA_MAX_LOAD;   // table load above which an end overflows (claims)
 
 // ---- shared-memory layout ------------------------------------------------------------------------
 // [info0: icap u32][info1: icap u32][walk strings: 4 x Wp][table region: B1 | B2 | keys | cnts]
@@ -1155,7 +1158,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                     const uint32_t code = inf & 7u;
                     if (code == CODE_FORK) { term = T_FORK; break; }
                     if (code == CODE_DEADEND) { term = T_DEADEND; break; }
-                    wb[len++] = "ACGT"[code];
+                    wb[len++] = (uint8_t)(0x54474341u >> (8 * code));   // "ACGT"[code] without a memory lookup
                     node = inf >> 4;
                 }
                 E.attempts += 1;
@@ -1576,7 +1579,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                     const uint32_t code = inf & 7u;
                     if (code == CODE_FORK) { term = T_FORK; break; }
                     if (code == CODE_DEADEND) { term = T_DEADEND; break; }
-                    wb[len++] = "ACGT"[code];
+                    wb[len++] = (uint8_t)(0x54474341u >> (8 * code));   // "ACGT"[code] without a memory lookup
                     node = inf >> 4;
                 }
                 E.attempts += 1;
