@@ -468,90 +468,6 @@ __device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq
     }
 }
 
-// Lane-per-run variant: warp iteration = 32*RUN consecutive positions, lane l takes the RUN positions
-// base + l*RUN + i.  The k-mer is extracted once per run (or when the run crosses into the next read)
-// and rolled (next_kmer, Alg 2 line 15) for the others, so a position costs a roll, not an extraction.
-// f(act, v) is called RUN times per iteration by the whole warp.
-template <int RUN, typename F>
-__device__ __forceinline__ void warp_runs(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
-                                          const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
-                                          int r, int SW, int k, int KW, int wid, int nwarps, int lane,
-                                          const volatile int *stop, F &&f) {
-    const uint32_t total = pref[r];
-    const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
-    const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
-    if (wb >= we) return;
-    uint64_t m0, m1;
-    kmer_masks(k, m0, m1);
-    constexpr uint32_t SPAN = 32u * RUN;
-    int j;
-    {   // read j with pref[j] <= g < pref[j+1]
-        const uint32_t gg = min(wb + (uint32_t)lane * RUN, we - 1);
-        int lo = 0, hi = r;
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (pref[mid] <= gg) lo = mid; else hi = mid;
-        }
-        j = lo;
-    }
-    uint32_t pj0 = pref[j], pj1 = pref[j + 1];
-    const uint64_t *R = rseq + (r0 + j) * SW, *Q = rqc + (r0 + j) * SW;
-    bool flag = rflag[r0 + j] != 0;
-    KmerN<2> K;
-    K.w[0] = K.w[1] = 0;
-    int p = 0, lastN = -1;
-    uint32_t g = wb + (uint32_t)lane * RUN;   // this lane's next position
-    for (uint32_t base = wb; base < we; base += SPAN) {
-        if (((base - wb) & (4u * SPAN - 1u)) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;
-        g = base + (uint32_t)lane * RUN;
-#pragma unroll 1
-        for (int i = 0; i < RUN; ++i, ++g) {
-            const bool act = g < we;
-            if (act && (i == 0 || g >= pj1)) {   // (re)start: run start or the run entered a later read
-                if (g >= pj1) {
-                    do {
-                        pj0 = pj1;
-                        pj1 = pref[++j + 1];
-                    } while (g >= pj1);
-                    R = rseq + (r0 + j) * SW;
-                    Q = rqc + (r0 + j) * SW;
-                    flag = rflag[r0 + j] != 0;
-                }
-                p = (int)(g - pj0);
-                const int q = p >> 5, sft = (p & 31) << 1, q2 = min(q + 2, SW - 1);
-                const uint64_t w0 = R[q], w1 = R[q + 1], w2 = R[q2];
-                K.w[0] = funnel64(w0, w1, sft) & m0;
-                K.w[1] = funnel64(w1, w2, sft) & m1;
-                lastN = -1;
-                if (flag) {   // last N inside the window [p, p+k) (bit 62-2i of nmask marks base i)
-                    const uint64_t n0 = nmask_word(Q[q]), n1 = nmask_word(Q[q + 1]), n2 = nmask_word(Q[q2]);
-                    const uint64_t N0 = funnel64(n0, n1, sft) & m0, N1 = funnel64(n1, n2, sft) & m1;
-                    lastN = N1 ? p + 32 + ((62 - (__ffsll((long long)N1) - 1)) >> 1)
-                               : (N0 ? p + ((62 - (__ffsll((long long)N0) - 1)) >> 1) : -1);
-                }
-            }
-            PosV v;
-            v.vote = false;
-            v.nb = 0;
-            v.hi = false;
-            if (act) {
-                const int ii = p + k, sh = 62 - ((ii & 31) << 1);
-                v.nb = (uint32_t)(R[ii >> 5] >> sh) & 3u;
-                const uint32_t nq = (uint32_t)(Q[ii >> 5] >> sh) & 3u;
-                v.vote = nq - 1u < 2u && lastN < p;
-                v.hi = nq == 2u;
-                if (nq == 3u) lastN = ii;
-            }
-            v.K = K;
-            f(act && v.vote, v);
-            if (act) {   // next_kmer (Alg 2 line 15) for the lane's next position
-                roll_kmer(K, k, KW, v.nb);
-                ++p;
-            }
-        }
-    }
-}
-
 // Convergent insert of the lanes with `want` (Alg 1 line 5 + the vote): every probe round
 // is entered by the whole warp and tests a slot pair (s, s+1); claims are counted once per warp.
 // One slot of a round: 0 = resolved (found or claimed), 1 = occupied by another key, 2 = gave up
@@ -925,19 +841,6 @@ __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
     return (code < 4 ? (nxt == NONE ? NEXT_NONE : nxt) : NEXT_NONE) << 4 | (uint32_t)code;
 }
 
-#ifndef LA_RUN
-#define LA_RUN 1   // positions per lane per warp iteration: 1 = warp_positions (measured fastest), >1 = warp_runs
-#endif
-template <typename F>
-__device__ __forceinline__ void warp_pass(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
-                                          const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
-                                          int r, int SW, int k, int KW, int wid, int nwarps, int lane,
-                                          const volatile int *stop, F &&f) {
-    if (LA_RUN > 1)
-        warp_runs<LA_RUN>(rseq, rqc, rflag, pref, r0, r, SW, k, KW, wid, nwarps, lane, stop, f);
-    else
-        warp_positions(rseq, rqc, rflag, pref, r0, r, SW, k, KW, wid, nwarps, lane, stop, f);
-}
 template <bool INL, bool GT>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
@@ -952,7 +855,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
     if (INL) {
         // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
         if (mbits) {
-            warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+            warp_positions(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
                            [&](bool act, const PosV &v) {
                                if (!act) return;
                                const uint32_t fi = filt_index(hash_kmer(v.K, KW), mbits);
@@ -967,7 +870,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
         t_filter = clock64();
         // ---- build (Alg 1) ----
         {
-            warp_pass(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+            warp_positions(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
                       [&](bool act, const PosV &v) {
                           const uint64_t h = hash_kmer(v.K, KW);
                           bool want = act;
