@@ -27,6 +27,19 @@
 namespace la {
 
 enum : int { CLS_NOREADS = 0, CLS_SHORT = 1, CLS_S = 2, CLS_GLOBAL = 8 };   // CLS_S + class index (5 = XL)
+// Phase clocks (tools/phase_profile.py builds with -DLA_PROFILE_CLOCKS=1): compiled out by default so
+// the per-phase cycle accumulators take no registers in the production kernels.
+#ifndef LA_PROFILE_CLOCKS
+#define LA_PROFILE_CLOCKS 0
+#endif
+__device__ __forceinline__ long long la_clock() {
+#if LA_PROFILE_CLOCKS
+    return clock64();
+#else
+    return 0;
+#endif
+}
+
 #ifndef LA_MAX_LOAD
 #define LA_MAX_LOAD 0.70f
 #endif
@@ -298,6 +311,8 @@ struct TabCtx {   // what a table operation needs
     uint64_t *keys;
     uint32_t *c32;   // per slot: word 0 = low-only votes[4] (8 bits each), word 1 = high votes[4]
     uint16_t *list;  // claimed slots in claim order (inline keys): the link pass visits only these
+    uint32_t ks;     // shared-memory address of keys (shared tables): computed once, so the probe
+                     // loops do not rematerialise the generic->shared conversion (S2R) every round
     uint32_t cap;
     const uint64_t *rseq;   // packed reads (global), for REF-format key verification
     int SW, k, KW;
@@ -336,6 +351,40 @@ __device__ __forceinline__ void votes_of(const TabCtx &T, uint32_t s, uint32_t l
 // Inline-key tables probe linearly from an even slot, so that a probe round can test the slot pair
 // (s, s+1) with two adjacent 16 B loads (cap is even).
 __device__ __forceinline__ uint32_t slot0_inl(uint64_t h, uint32_t cap) { return slot_of(h, cap) & ~1u; }
+
+template <bool GT>
+__device__ __forceinline__ void slot_ld128(const TabCtx &T, size_t s, uint64_t &x, uint64_t &y) {
+    if (GT)
+        asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(x), "=l"(y) : "l"(T.keys + 2 * s) : "memory");
+    else
+        asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];"
+                     : "=l"(x), "=l"(y)
+                     : "r"(T.ks + 16u * (uint32_t)s)
+                     : "memory");
+}
+template <bool GT>
+__device__ __forceinline__ void slot_cas128(const TabCtx &T, size_t s, uint64_t n0, uint64_t n1, uint64_t &o0,
+                                            uint64_t &o1) {
+    if (GT) {
+        cas128<true>((void *)(T.keys + 2 * s), 0ull, 0ull, n0, n1, o0, o1);
+    } else {
+        asm volatile(
+            "{\n .reg .b128 d, b, c;\n mov.b128 b, {%2, %3};\n mov.b128 c, {%4, %5};\n"
+            " atom.shared.cas.b128 d, [%6], b, c;\n mov.b128 {%0, %1}, d;\n}"
+            : "=l"(o0), "=l"(o1)
+            : "l"(0ull), "l"(0ull), "l"(n0), "l"(n1), "r"(T.ks + 16u * (uint32_t)s)
+            : "memory");
+    }
+}
+template <bool GT>
+__device__ __forceinline__ uint64_t slot_ld_w0(const TabCtx &T, size_t s) {
+    uint64_t x;
+    if (GT)
+        asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(x) : "l"(T.keys + 2 * s) : "memory");
+    else
+        asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(x) : "r"(T.ks + 16u * (uint32_t)s) : "memory");
+    return x;
+}
 
 template <bool INL, int NW>
 __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> &K, uint64_t h) {
@@ -477,17 +526,17 @@ __device__ __forceinline__ int probe_slot(const TabCtx &T, uint32_t s, uint64_t 
                                           bool &claimed, volatile int *ovf) {
     if (y == 0) {   // looks empty: the CAS claims it or returns its true content
         if (*ovf) return 2;
-        cas128<GT>((void *)&T.keys[2 * (size_t)s], 0ull, 0ull, a, bb, x, y);
+        slot_cas128<GT>(T, s, a, bb, x, y);
         if (y == 0) {
             claimed = true;
             return 0;
         }
-        if (y == bb && x != a) x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
+        if (y == bb && x != a) x = slot_ld_w0<GT>(T, s);
         return (x == a && y == bb) ? 0 : 3;
     }
     // a 16 B load is not single-copy atomic: if it raced with the claiming CAS, word 0 may be stale —
     // re-read it (a slot never changes once claimed)
-    if (y == bb && x != a) x = *(volatile uint64_t *)&T.keys[2 * (size_t)s];
+    if (y == bb && x != a) x = slot_ld_w0<GT>(T, s);
     return (x == a && y == bb) ? 0 : 1;
 }
 
@@ -507,8 +556,8 @@ __device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const Po
         if (pend) {
             uint64_t x0, y0, x1, y1;
             const uint32_t s1 = s + 1 == T.cap ? 0 : s + 1;   // s is even except after a lost claim race
-            ld128v<GT>(&T.keys[2 * (size_t)s], x0, y0);
-            ld128v<GT>(&T.keys[2 * (size_t)s1], x1, y1);
+            slot_ld128<GT>(T, s, x0, y0);
+            slot_ld128<GT>(T, s1, x1, y1);
             int st = probe_slot<GT>(T, s, x0, y0, a, bb, claimed, ovf);
             if (st == 0) {
                 hit = s;
@@ -714,8 +763,8 @@ __device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, cons
         if ((threadIdx.x & 31) == 0) LA_PSTAT(5, 1);
         if (pend) {
             uint64_t x0, y0, x1, y1;
-            ld128v<GT>(&T.keys[2 * (size_t)s], x0, y0);
-            ld128v<GT>(&T.keys[2 * (size_t)s + 2], x1, y1);   // s even, cap even: s+1 < cap
+            slot_ld128<GT>(T, s, x0, y0);
+            slot_ld128<GT>(T, s + 1, x1, y1);   // s even, cap even: s+1 < cap
             if (y0 == 0) {
                 pend = false;
             } else if (x0 == a && y0 == bb) {
@@ -867,7 +916,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                            });
             builders_sync(NB);
         }
-        t_filter = clock64();
+        t_filter = la_clock();
         // ---- build (Alg 1) ----
         {
             warp_positions(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
@@ -896,7 +945,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                });
             builders_sync(NB);
         }
-        t_filter = clock64();
+        t_filter = la_clock();
         warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
                            [&](bool act, const PosR &v) {
                                const uint64_t h = hash_kmer(v.K, KW);
@@ -909,7 +958,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                            });
     }
     builders_sync(NB);
-    t_build = clock64();
+    t_build = la_clock();
     if (B.overflow) return;
 #ifdef LA_PROBE_STATS
     if (bt == 0) LA_PSTAT(7, (unsigned long long)B.nclaim * 1000ull / T.cap);
@@ -1001,6 +1050,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     __shared__ EndSlot S[2];
     __shared__ BuildCtl B;
     __shared__ __align__(8) uint64_t built[2], walked[2];   // mbarriers: slot s built / walked
+    __shared__ unsigned long long s_acc[4];   // work counters: inserts, walk steps, attempts, filtered
     const int tid = threadIdx.x;
     const SmemFixed FX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u);
     // table region: shared memory, or this CTA's slice of the global scratch (XL class)
@@ -1015,6 +1065,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             S[i].dead = 0;
             S[i].ovf = 0;
         }
+        for (int i = 0; i < 4; ++i) s_acc[i] = 0;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -1024,14 +1075,14 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     if (tid < 32) {
         // ============================ walker warp ============================
         const int lane = tid;
-        unsigned long long acc_ins = 0, acc_steps = 0, acc_att = 0;
+
         uint32_t phase = 0u, alive = 3u;   // bit s: mbarrier parity / slot still in use
         long long w_wait = 0, w_walk = 0;
         for (int s = 0; alive; s ^= 1) {
             if (!((alive >> s) & 1u)) continue;
-            const long long tw0 = clock64();
+            const long long tw0 = la_clock();
             if (lane == 0) mbar_wait(&built[s], (phase >> s) & 1u);
-            w_wait += clock64() - tw0;
+            w_wait += la_clock() - tw0;
             phase ^= 1u << s;
             __syncwarp();
             EndSlot &E = S[s];
@@ -1044,7 +1095,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                 continue;
             }
             int done = 0, bl = 0, bb = 0;
-            const long long tw1 = clock64();
+            const long long tw1 = la_clock();
             if (lane == 0) {
                 // ---- walk (Alg 2) over the successor links ----
                 uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
@@ -1082,7 +1133,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             done = __shfl_sync(0xffffffffu, done, 0);
             bl = __shfl_sync(0xffffffffu, bl, 0);
             bb = __shfl_sync(0xffffffffu, bb, 0);
-            w_walk += clock64() - tw1;
+            w_walk += la_clock() - tw1;
             if (done) {
                 // ---- the selected walk -> HBM ----
                 const int e = E.e;
@@ -1094,9 +1145,9 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                     out_term[e] = (uint8_t)E.best_term;
                     out_k[e] = (uint8_t)E.best_k;
                     out_att[e] = (uint8_t)E.attempts;
-                    acc_ins += E.ins;
-                    acc_steps += E.steps;
-                    acc_att += E.attempts;
+                    s_acc[0] += E.ins;   // per-CTA work counters in shared memory (no registers)
+                    s_acc[1] += E.steps;
+                    s_acc[2] += E.attempts;
                     E.done = 1;
                 }
             }
@@ -1104,9 +1155,9 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             if (lane == 0) mbar_arrive(&walked[s]);   // release: the state above is visible to the builders
         }
         if (lane == 0) {
-            atomicAdd(&gstats->inserts, acc_ins);
-            atomicAdd(&gstats->steps, acc_steps);
-            atomicAdd(&gstats->attempts, acc_att);
+            atomicAdd(&gstats->inserts, s_acc[0]);
+            atomicAdd(&gstats->steps, s_acc[1]);
+            atomicAdd(&gstats->attempts, s_acc[2]);
             if (prof) {
                 atomicAdd(&prof[6], (unsigned long long)w_wait);
                 atomicAdd(&prof[7], (unsigned long long)w_walk);
@@ -1118,12 +1169,11 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
     // ============================ builders ============================
     const int bt = tid - 32;
     uint32_t wphase = 0u, first = 3u, alive = 3u;   // bit s; alive is identical in every builder
-    unsigned long long n_filtered = 0;
     long long b_t[6] = {0, 0, 0, 0, 0, 0};   // builder-leader cycles: wait, prefix, clear, filter, build, link
     for (int s = 0; alive; s ^= 1) {
         if (!((alive >> s) & 1u)) continue;
         EndSlot &E = S[s];
-        const long long ta = clock64();
+        const long long ta = la_clock();
         if (bt == 0) {
             if (!((first >> s) & 1u)) {
                 mbar_wait(&walked[s], (wphase >> s) & 1u);   // acquire: the walker's update of slot s
@@ -1161,7 +1211,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             }
         }
         builders_sync(NB);
-        const long long tb = clock64();
+        const long long tb = la_clock();
         b_t[0] += tb - ta;
         if (B.skip) {
             alive &= ~(1u << s);
@@ -1210,7 +1260,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
             read_prefix(B, E, pref, gL, lr0, r, k, ulen, bt, NB);
         }
         const uint32_t U = no_room ? 0u : pref[r];
-        const long long tc = clock64();
+        const long long tc = la_clock();
         b_t[1] += tc - tb;
         long long td = tc, t_filter = tc, t_build = tc;
         // XL: stage this end's reads in shared memory when they fit beside the filter bitmaps (the
@@ -1257,13 +1307,14 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         bool ovf = no_room || TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
         if (!ovf) {
             const uint32_t mbits = TB.mwords * 32u;
-            if (mbits) ++n_filtered;
+            if (mbits && bt == 0) s_acc[3] += 1;
             uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);   // filters: always shared memory
             uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
             TabCtx T;
             T.keys = (uint64_t *)(tbase + TB.off_keys);
             T.c32 = (uint32_t *)(tbase + TB.off_cnts);
             T.list = (uint16_t *)(tbase + TB.off_list);
+            T.ks = GT ? 0u : (uint32_t)__cvta_generic_to_shared(T.keys);
             T.cap = TB.cap;
             T.rseq = gR;   // REF keys store read indices relative to gR
             T.SW = SW;
@@ -1278,7 +1329,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
                 for (uint32_t i = bt; i < 2u * TB.mwords; i += NB) B1[i] = 0;   // B1, B2 contiguous
             }
             builders_sync(NB);
-            td = clock64();
+            td = la_clock();
             t_filter = t_build = td;
             const int e = E.e;
             const int Tn = min((int)clen[e], 128);
@@ -1295,7 +1346,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         }
         builders_sync(NB);   // info buffer complete; the table is free for the next build
         {
-            const long long te = clock64();
+            const long long te = la_clock();
             b_t[2] += td - tc;
             b_t[3] += t_filter - td;
             b_t[4] += t_build - t_filter;
@@ -1316,7 +1367,7 @@ __global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_sm
         }
     }
     if (bt == 0) {
-        atomicAdd(&gstats->filtered, n_filtered);
+        atomicAdd(&gstats->filtered, s_acc[3]);
         if (prof)
             for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
     }
@@ -1349,15 +1400,16 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
     __shared__ EndSlot E;
     __shared__ BuildCtl B;
     __shared__ int s_done;
+    __shared__ unsigned long long s_acc[4];   // work counters: inserts, walk steps, attempts, filtered
     const int bt = threadIdx.x;
     const SmemFixed FX = smem_fixed(P.W, smem_bytes, 0u, true);
     const int Wp = (P.W + 15) & ~15;
     uint8_t *wstr = sm + FX.off_walk;   // two walk strings: current / best
     uint32_t *info = (uint32_t *)sm;
-    unsigned long long acc_ins = 0, acc_steps = 0, acc_att = 0, n_filtered = 0;
+    if (bt < 4) s_acc[bt] = 0;   // published by the first __syncthreads below
     long long b_t[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // leader cycles: fetch, prefix, clear, filter, build, link, -, walk
     for (;;) {
-        const long long ta = clock64();
+        const long long ta = la_clock();
         if (bt == 0) {
             const int idx = atomicAdd(work_ctr, 1);
             B.skip = idx >= n_list;
@@ -1409,9 +1461,9 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
         const uint64_t *tail_e = tail + (size_t)e * TAIL_W;
         const uint64_t n0 = tailN[2 * (size_t)e], n1 = tailN[2 * (size_t)e + 1];
         __syncthreads();
-        b_t[0] += clock64() - ta;
+        b_t[0] += la_clock() - ta;
         while (!ovf) {   // attempts (k schedule)
-            const long long tb = clock64();
+            const long long tb = la_clock();
             const int k = E.k;
             const int KW = kwords(k);
             read_prefix(B, E, pref, sL, 0, r, k, E.ulen, bt, NB);
@@ -1422,13 +1474,14 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 break;
             }
             const uint32_t mbits = TB.mwords * 32u;
-            if (mbits) ++n_filtered;
+            if (mbits && bt == 0) s_acc[3] += 1;
             uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);
             uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
             TabCtx T;
             T.keys = (uint64_t *)(sm + TB.off_keys);
             T.c32 = (uint32_t *)(sm + TB.off_cnts);
             T.list = (uint16_t *)(sm + TB.off_list);
+            T.ks = (uint32_t)__cvta_generic_to_shared(T.keys);
             T.cap = TB.cap;
             T.rseq = sR;
             T.SW = SW;
@@ -1438,7 +1491,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 B.overflow = 0;
                 B.nclaim = 0;
             }
-            const long long tc = clock64();
+            const long long tc = la_clock();
             {
                 const uint4 z = make_uint4(0, 0, 0, 0);
                 uint4 *a = (uint4 *)T.keys;
@@ -1447,7 +1500,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 for (uint32_t i = bt; i < 2u * TB.mwords; i += NB) B1[i] = 0;
             }
             __syncthreads();
-            const long long td = clock64();
+            const long long td = la_clock();
             long long t_filter = td, t_build = td;
             if (inline_keys(k))
                 build_link<true, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
@@ -1456,7 +1509,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
                                          NB, t_filter, t_build);
             __syncthreads();
-            const long long te = clock64();
+            const long long te = la_clock();
             b_t[1] += tc - tb;
             b_t[2] += td - tc;
             b_t[3] += t_filter - td;
@@ -1499,7 +1552,7 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 E.shift = sh;
             }
             __syncthreads();
-            b_t[7] += clock64() - te;
+            b_t[7] += la_clock() - te;
             if (s_done) break;
         }
         if (ovf) {   // table or counter overflow: the global path redoes this end from scratch
@@ -1514,18 +1567,18 @@ __global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
                 out_term[e] = (uint8_t)E.best_term;
                 out_k[e] = (uint8_t)E.best_k;
                 out_att[e] = (uint8_t)E.attempts;
-                acc_ins += E.ins;
-                acc_steps += E.steps;
-                acc_att += E.attempts;
+                s_acc[0] += E.ins;
+                s_acc[1] += E.steps;
+                s_acc[2] += E.attempts;
             }
         }
         __syncthreads();   // E and the staged reads are reused by the next end
     }
     if (bt == 0) {
-        atomicAdd(&gstats->inserts, acc_ins);
-        atomicAdd(&gstats->steps, acc_steps);
-        atomicAdd(&gstats->attempts, acc_att);
-        atomicAdd(&gstats->filtered, n_filtered);
+        atomicAdd(&gstats->inserts, s_acc[0]);
+        atomicAdd(&gstats->steps, s_acc[1]);
+        atomicAdd(&gstats->attempts, s_acc[2]);
+        atomicAdd(&gstats->filtered, s_acc[3]);
         if (prof) {
             for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
             atomicAdd(&prof[7], (unsigned long long)b_t[7]);

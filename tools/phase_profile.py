@@ -1,4 +1,5 @@
-"""Per-class phase breakdown of the shared-memory kernels (LA_PROFILE=1 clock64 counters).
+"""Per-class phase breakdown of the shared-memory kernels (clock64 counters: builds a copy of the
+library with -DLA_PROFILE_CLOCKS=1 and runs it with LA_PROFILE=1).
 
   python tools/phase_profile.py [--config C4] [--scale 1.0]
 Prints, per table class, the builders' leader cycles split into wait / prefix / clear / filter /
@@ -19,6 +20,15 @@ def main():
     ap.add_argument("--scale", type=float, default=1.0)
     a = ap.parse_args()
     os.environ["LA_PROFILE"] = "1"
+    # the phase clocks are compiled out of the production library: build a profiling copy
+    import importlib.util
+    import subprocess
+    so = "/tmp/liblocassm_prof.so"
+    os.environ["LA_SO"] = so   # before the package (and its ctypes binding) is imported
+    spec = importlib.util.spec_from_file_location("la_build", os.path.join(ROOT, "paper_conf_sc_awanhedbdoy21_b200", "build.py"))
+    b = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(b)
+    subprocess.check_call([b.NVCC, *b.FLAGS, "-DLA_PROFILE_CLOCKS=1", "-o", so, *b.SRC])
     import bench
     from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
     batch, params = bench.load_workload(a.config, 0, a.scale)
