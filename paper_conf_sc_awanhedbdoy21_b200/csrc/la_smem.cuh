@@ -1033,8 +1033,9 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
     }
 }
 
-template <int BLOCK, bool GT>
-__global__ void __launch_bounds__(BLOCK, 768 / BLOCK > 0 ? 768 / BLOCK : 1) k_smem(
+// MINB: resident CTAs per SM the class is launched with (register budget 65536 / (MINB * BLOCK))
+template <int BLOCK, bool GT, int MINB = (768 / BLOCK > 0 ? 768 / BLOCK : 1)>
+__global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     const int32_t *__restrict__ list, int n_list, int *__restrict__ work_ctr,
     const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
     const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,

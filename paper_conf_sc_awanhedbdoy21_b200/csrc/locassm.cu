@@ -248,6 +248,7 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         attr_ok &= cudaFuncSetAttribute(k_smem<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_smem<192, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        attr_ok &= cudaFuncSetAttribute(k_smem<256, false, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_small<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
         attr_ok &= cudaFuncSetAttribute(k_small<96>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
@@ -720,7 +721,18 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
                     case 96: LA_LAUNCH_SMEM(96); break;
                     case 192: LA_LAUNCH_SMEM(192); break;
                     case 128: LA_LAUNCH_SMEM(128); break;
-                    case 256: LA_LAUNCH_SMEM(256); break;
+                    case 256:
+                        if (ctx->cls_ctas[c] <= 2) {   // 2 CTAs/SM: a 128-register budget
+                            k_smem<256, false, 2><<<grid, 256, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq),
+                                P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff),
+                                P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
+                                P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term),
+                                P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,
+                                (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr);
+                        } else {
+                            LA_LAUNCH_SMEM(256);
+                        }
+                        break;
                     default: LA_LAUNCH_SMEM(512); break;
                 }
             }
