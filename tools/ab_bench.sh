@@ -1,4 +1,8 @@
 set -e
+# Usage: populate _headcsrc/ (git-ignored) with the HEAD sources first, e.g.
+#   mkdir -p _headcsrc/csrc _headcsrc/include; for f in la_device.cuh la_global.cuh la_kernels.cuh la_smem.cuh locassm.cu; do
+#     git show HEAD:paper_conf_sc_awanhedbdoy21_b200/csrc/$f > _headcsrc/csrc/$f; done; git show HEAD:include/locassm.h > _headcsrc/include/locassm.h
+# then: gpurun -- bash tools/ab_bench.sh
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -shared -Xcompiler -fPIC -I_headcsrc/include -o /tmp/head.so _headcsrc/csrc/locassm.cu
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -shared -Xcompiler -fPIC -Iinclude -DLA_CLAIM_PTX=1 -o /tmp/ptx.so paper_conf_sc_awanhedbdoy21_b200/csrc/locassm.cu
