@@ -406,7 +406,7 @@ def main():
                                  "attempts": st["cls_attempts"][i], "filtered": st["cls_filtered"][i],
                                  "ms": round(st["cls_ms"][i], 3)}
                              for i, n in enumerate(["smem64x12", "smem128x6", "smem256x3", "smem256x2",
-                                                    "smem512x1", "xl512x1"])}},
+                                                    "smem1024x1", "xl512x1"])}},
         "roofline": roof,
         "roofline_insert": ({"bound": "smem", "kernel": roof["kernel"], "achieved": roof["achieved"],
                              "peak": peaks["insert_gups"], "unit": "G inserts/s",

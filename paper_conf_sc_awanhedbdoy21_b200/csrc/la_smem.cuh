@@ -178,7 +178,7 @@ __device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, u
 }
 
 // Shared-memory classes, smallest CTA first: (threads, CTAs/SM) = (64, 12), (128, 6), (256, 3),
-// (256, 2), (512, 1); one warp of each CTA walks, the others build.  The first class whose table is
+// (256, 2), (1024, 1); one warp of each CTA walks, the others build.  The first class whose table is
 // predicted to fit wins; G = global-memory rounds.
 constexpr int N_SMEM_CLASSES = 5;
 struct PlanBytes {
@@ -801,7 +801,7 @@ struct BuildCtl {           // builders' shared scratch
     int overflow, nclaim;
     uint32_t start;
     int lmin, lmax;
-    uint32_t wsum[16];      // per builder warp: prefix-scan totals
+    uint32_t wsum[32];      // per builder warp: prefix-scan totals
 };
 
 __device__ __forceinline__ void builders_sync(int NB) { asm volatile("bar.sync 1, %0;" ::"r"(NB) : "memory"); }
