@@ -191,7 +191,10 @@ __host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { r
 
 // XL class: 512-thread CTAs (1 per SM) whose tables live in a per-CTA global-memory scratch (L2-resident
 // for the paper-shaped batch); shared memory keeps the info buffers (so the walk stays on-chip).
-constexpr int XL_THREADS = 512;
+#ifndef LA_XL_THREADS
+#define LA_XL_THREADS 1024   // 1024 vs 768 vs 512 threads: 154 / 156 / 162 ms on C4 (r01)
+#endif
+constexpr int XL_THREADS = LA_XL_THREADS;
 constexpr int64_t XL_MAX_U = 1 << 21;
 __host__ __device__ __forceinline__ uint32_t xl_needed_cap(int64_t r, int64_t U, bool filter) {
     const float need = filter ? (filtered_fraction(r) * (float)U + 1024.f) : (float)U;
@@ -200,6 +203,7 @@ __host__ __device__ __forceinline__ uint32_t xl_needed_cap(int64_t r, int64_t U,
 // bytes of one CTA's global scratch for the largest XL end (U_max occurrences, r_max reads)
 __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_max, bool filter, uint32_t icap) {
     uint32_t cap = xl_needed_cap(r_max, U_max, filter);
+    if (cap < min_table_cap(XL_THREADS)) cap = min_table_cap(XL_THREADS);   // claims + in-flight < cap
     if (cap > icap) cap = icap;
     return (pref_bytes((int)r_max) + 32u + cap * (16u + cnt_bytes(true) + 2u) + 255u) & ~255u;
 }
@@ -1298,7 +1302,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
         }
         SmemTab TB = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW);
         if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
-            const uint32_t need = xl_needed_cap(r, U, TB.mwords != 0);
+            const uint32_t need = max(xl_needed_cap(r, U, TB.mwords != 0), min_table_cap(BLOCK));
             if (TB.cap > need) {
                 TB.cap = (need + 1u) & ~1u;
                 TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
