@@ -405,8 +405,8 @@ def main():
                  "classes": {n: {"ends": st["cls_ends"][i], "inserts": st["cls_inserts"][i],
                                  "attempts": st["cls_attempts"][i], "filtered": st["cls_filtered"][i],
                                  "ms": round(st["cls_ms"][i], 3)}
-                             for i, n in enumerate(["smem64x12", "smem128x6", "smem256x3", "smem256x2",
-                                                    "smem1024x1", "xl512x1"])}},
+                             for i, n in enumerate(["smem64x12", "smem128x6", "smem256x3", "smem512x2",
+                                                    "smem1024x1", "xl1024x1"])}},
         "roofline": roof,
         "roofline_insert": ({"bound": "smem", "kernel": roof["kernel"], "achieved": roof["achieved"],
                              "peak": peaks["insert_gups"], "unit": "G inserts/s",

@@ -178,7 +178,7 @@ __device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, u
 }
 
 // Shared-memory classes, smallest CTA first: (threads, CTAs/SM) = (64, 12), (128, 6), (256, 3),
-// (256, 2), (1024, 1); one warp of each CTA walks, the others build.  The first class whose table is
+// (512, 2), (1024, 1); one warp of each CTA walks, the others build.  The first class whose table is
 // predicted to fit wins; G = global-memory rounds.
 constexpr int N_SMEM_CLASSES = 5;
 struct PlanBytes {
@@ -1378,17 +1378,15 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     }
 }
 
-#ifndef LA_SMALL_MINB
-#define LA_SMALL_MINB(B) (768 / (B) > 0 ? 768 / (B) : 1)
-#endif
+
 // ---- k_small: one end per CTA, every thread builds, thread 0 walks -------------------------------
 // For the small-table classes the walk (a few thousand cycles) is short next to the build, so a
 // dedicated walker warp only halves the warps that build (ncu: the builders are latency-bound at
 // ~2 warps/SMSP).  Here all BLOCK threads build; after the link pass thread 0 walks while the others
 // wait at the barrier (other CTAs on the SM keep the issue slots busy).  The reads are staged in
 // shared memory once per end (not per attempt).
-template <int BLOCK>
-__global__ void __launch_bounds__(BLOCK, LA_SMALL_MINB(BLOCK)) k_small(
+template <int BLOCK, int MINB = (768 / BLOCK > 0 ? 768 / BLOCK : 1)>
+__global__ void __launch_bounds__(BLOCK, MINB) k_small(
     const int32_t *__restrict__ list, int n_list, int *__restrict__ work_ctr,
     const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
     const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,

@@ -53,6 +53,35 @@ struct Encoded {
 
 }  // namespace
 
+namespace {
+// Table-class kernels by (threads, resident CTAs per SM, k_small?): the launch bound gives each
+// instantiation the register budget 65536 / (threads x CTAs).  LA_CLASSES picks among these.
+using ClassKernel = void (*)(const int32_t *, int, int *, const uint64_t *, const uint64_t *, const uint16_t *,
+                             const uint8_t *, const int64_t *, const uint64_t *, const uint64_t *, const int32_t *,
+                             int, DevParams, uint32_t, uint8_t *, int32_t *, uint8_t *, uint8_t *, uint8_t *,
+                             int32_t *, int *, GlobalStats *, unsigned char *, uint32_t, unsigned long long *);
+struct ClassEntry {
+    int threads, ctas;
+    bool small;
+    ClassKernel fn;
+};
+const ClassEntry kClassKernels[] = {
+    {64, 12, true, k_small<64, 12>},     {64, 16, true, k_small<64, 16>},     {96, 8, true, k_small<96, 8>},
+    {128, 6, true, k_small<128, 6>},     {128, 8, true, k_small<128, 8>},     {192, 4, true, k_small<192, 4>},
+    {256, 3, true, k_small<256, 3>},     {256, 4, true, k_small<256, 4>},
+    {128, 6, false, k_smem<128, false, 6>}, {192, 4, false, k_smem<192, false, 4>},
+    {256, 3, false, k_smem<256, false, 3>}, {256, 2, false, k_smem<256, false, 2>},
+    {256, 4, false, k_smem<256, false, 4>}, {384, 2, false, k_smem<384, false, 2>},
+    {512, 2, false, k_smem<512, false, 2>}, {512, 1, false, k_smem<512, false, 1>},
+    {1024, 1, false, k_smem<1024, false, 1>},
+};
+const ClassEntry *find_class_kernel(int threads, int ctas, bool small) {
+    for (const ClassEntry &k : kClassKernels)
+        if (k.threads == threads && k.ctas == ctas && k.small == small) return &k;
+    return nullptr;
+}
+}  // namespace
+
 struct la_ctx {
     int device = 0;
     cudaStream_t stream = nullptr;
@@ -61,7 +90,7 @@ struct la_ctx {
     bool loaded = false;
     std::string err;
     int n_sm = 148;
-    int cls_threads[N_SMEM_CLASSES] = {64, 128, 256, 256, 1024};   // 1024x1 vs 512x1: 162 vs 166 ms (r01)
+    int cls_threads[N_SMEM_CLASSES] = {64, 128, 256, 512, 1024};   // r01: 256x2 -> 512x2 155 -> 146 ms, 512x1 -> 1024x1 166 -> 162 ms
     int cls_ctas[N_SMEM_CLASSES] = {12, 6, 3, 2, 1};   // resident CTAs per SM of each shared-memory class
     uint32_t cls_bytes[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};   // dynamic shared memory per CTA
     uint32_t xl_bytes = 0;        // dynamic shared memory of the XL class (the rest of the SM's 228 KB is L1)
@@ -186,22 +215,41 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     cudaDeviceProp prop;
     cudaGetDeviceProperties(&prop, device);
     ctx->n_sm = prop.multiProcessorCount;
-    // tuning hook: LA_CLASSES="64x12,128x6,256x3,256x2,512x1" (threads x CTAs/SM per class)
-    if (const char *cfg = getenv("LA_CLASSES")) {
-        int t, c, n = 0;
-        const char *q = cfg;
-        while (n < N_SMEM_CLASSES && sscanf(q, "%dx%d", &t, &c) == 2) {
-            if (t == 64 || t == 96 || t == 128 || t == 192 || t == 256 || t == 512 || t == 1024) {
-                ctx->cls_threads[n] = t;
-                ctx->cls_ctas[n] = std::max(1, c);
+    // tuning hook: LA_CLASSES="64x12,128x6,256x3,512x2,1024x1" (threads x CTAs/SM per class) and
+    // LA_SMALL_MASK (bit i: class i runs k_small); a combination without a kernel instantiation
+    // (kClassKernels) leaves the defaults in place
+    {
+        int th[N_SMEM_CLASSES], ct[N_SMEM_CLASSES];
+        uint32_t mask = ctx->small_mask;
+        for (int i = 0; i < N_SMEM_CLASSES; ++i) {
+            th[i] = ctx->cls_threads[i];
+            ct[i] = ctx->cls_ctas[i];
+        }
+        if (const char *cfg = getenv("LA_CLASSES")) {
+            int t, c, n = 0;
+            const char *q = cfg;
+            while (n < N_SMEM_CLASSES && sscanf(q, "%dx%d", &t, &c) == 2) {
+                th[n] = t;
+                ct[n] = std::max(1, c);
+                ++n;
+                q = strchr(q, ',');
+                if (!q) break;
+                ++q;
             }
-            ++n;
-            q = strchr(q, ',');
-            if (!q) break;
-            ++q;
+        }
+        if (const char *m = getenv("LA_SMALL_MASK")) mask = (uint32_t)strtoul(m, nullptr, 0);
+        bool ok = true;
+        for (int i = 0; i < N_SMEM_CLASSES; ++i) ok &= find_class_kernel(th[i], ct[i], (mask >> i) & 1u) != nullptr;
+        if (ok) {
+            for (int i = 0; i < N_SMEM_CLASSES; ++i) {
+                ctx->cls_threads[i] = th[i];
+                ctx->cls_ctas[i] = ct[i];
+            }
+            ctx->small_mask = mask;
+        } else {
+            fprintf(stderr, "locassm: LA_CLASSES / LA_SMALL_MASK names a class without a kernel; using defaults\n");
         }
     }
-    if (const char *m = getenv("LA_SMALL_MASK")) ctx->small_mask = (uint32_t)strtoul(m, nullptr, 0);
     // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
     for (int i = 0; i < N_SMEM_CLASSES; ++i) {
         size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - 512 /* static */;
@@ -243,20 +291,8 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     {
         uint32_t mx = 0;
         for (int i = 0; i < N_SMEM_CLASSES; ++i) mx = std::max(mx, ctx->cls_bytes[i]);
-        attr_ok &= cudaFuncSetAttribute(k_smem<64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<96, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<128, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<192, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<256, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<256, false, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<512, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_smem<1024, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<96>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<192>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
-        attr_ok &= cudaFuncSetAttribute(k_small<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
+        for (const ClassEntry &k : kClassKernels)
+            attr_ok &= cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
     }
     if (!attr_ok) {
         cudaGetLastError();
@@ -691,55 +727,13 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
             const uint32_t bytes = ctx->cls_bytes[c];
             int32_t *lst = lists + (size_t)c * nE;
             int *wc = d_ctr + 16 + c;
-#define LA_LAUNCH_SMEM(B)                                                                                   \
-    k_smem<B, false><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), \
-                                      P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail),             \
-                                      P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                 \
-                                      P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                       \
-                                      P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                         \
-                                      P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,                          \
-                                      (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr)
-#define LA_LAUNCH_SMALL(B)                                                                                  \
-    k_small<B><<<grid, B, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen),  \
-                                       P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail),            \
-                                       P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,                \
-                                       P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),                      \
-                                       P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),                        \
-                                       P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,                         \
-                                       (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr)
-            if ((ctx->small_mask >> c) & 1u) {
-                switch (ctx->cls_threads[c]) {
-                    case 64: LA_LAUNCH_SMALL(64); break;
-                    case 96: LA_LAUNCH_SMALL(96); break;
-                    case 192: LA_LAUNCH_SMALL(192); break;
-                    case 128: LA_LAUNCH_SMALL(128); break;
-                    case 256: LA_LAUNCH_SMALL(256); break;
-                    default: LA_LAUNCH_SMALL(512); break;
-                }
-            } else {
-                switch (ctx->cls_threads[c]) {
-                    case 64: LA_LAUNCH_SMEM(64); break;
-                    case 96: LA_LAUNCH_SMEM(96); break;
-                    case 192: LA_LAUNCH_SMEM(192); break;
-                    case 128: LA_LAUNCH_SMEM(128); break;
-                    case 256:
-                        if (ctx->cls_ctas[c] <= 2) {   // 2 CTAs/SM: a 128-register budget
-                            k_smem<256, false, 2><<<grid, 256, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq),
-                                P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff),
-                                P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
-                                P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term),
-                                P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,
-                                (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr);
-                        } else {
-                            LA_LAUNCH_SMEM(256);
-                        }
-                        break;
-                    case 1024: LA_LAUNCH_SMEM(1024); break;
-                    default: LA_LAUNCH_SMEM(512); break;
-                }
-            }
-#undef LA_LAUNCH_SMEM
-#undef LA_LAUNCH_SMALL
+const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], (ctx->small_mask >> c) & 1u);
+            if (!ke) return fail(ctx, LA_ERR_STATE, "no kernel instantiation for table class %d", c);
+            ke->fn<<<grid, ke->threads, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
+                P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
+                P<int32_t>(E.clen), E.SW, dp, bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+                P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,
+                (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr);
             CKL();
         }
         CK(cudaEventRecord(ctx->ev_cls[c], cls_st(c)));   // end of class c

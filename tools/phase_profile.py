@@ -37,7 +37,7 @@ def main():
         la.extend_device()
         la.extend_device()
         st = la.stats()
-    names = ["smem64x12", "smem128x6", "smem256x3", "smem256x2", "smem1024x1", "xl512x1"]
+    names = ["smem64x12", "smem128x6", "smem256x3", "smem512x2", "smem1024x1", "xl1024x1"]
     out = {}
     for c, n in enumerate(names):
         p = st["prof_cycles"][c]
