@@ -51,14 +51,20 @@ def main():
     names = re.findall(r"^\.text\.(\S+):$", sass, re.M)
     want = None
     short = re.sub(r"\(.*", "", kname.replace("void ", ""))
-    tmpl = re.search(r"<\(int\)(\d+), \(bool\)(\d)>", kname)
-    tsmall = re.search(r"k_small<\(int\)(\d+)>", kname)
+    tmpl = re.search(r"<\(int\)(\d+), \(bool\)(\d)(?:, \(int\)(\d+))?>", kname)
+    tsmall = re.search(r"k_small<\(int\)(\d+)(?:, \(int\)(\d+))?>", kname)
     for n in names:
         if "k_smem" in short and tmpl:
-            if n.startswith("_ZN2la6k_smemILi%sELb%s" % (tmpl.group(1), tmpl.group(2))):
+            pre = "_ZN2la6k_smemILi%sELb%sE" % (tmpl.group(1), tmpl.group(2))
+            if tmpl.group(3):
+                pre += "Li%sE" % tmpl.group(3)
+            if n.startswith(pre):
                 want = n
         elif tsmall:
-            if n.startswith("_ZN2la7k_smallILi%sE" % tsmall.group(1)):
+            pre = "_ZN2la7k_smallILi%sE" % tsmall.group(1)
+            if tsmall.group(2):
+                pre += "Li%sE" % tsmall.group(2)
+            if n.startswith(pre):
                 want = n
         elif short.split("::")[-1] in n:
             want = want or n
