@@ -139,6 +139,20 @@ la_status la_extend_device(la_ctx *ctx, la_result *out);
  * la_load_batch, the context's loaded batch is then unspecified until the next la_load_batch). */
 la_status la_extend_streamed(la_ctx *ctx, const la_batch *batch, const la_params *params, int32_t n_chunks,
                              la_result *out);
+/* On-device append of extensions to contigs (the "Append extensions to contigs"
+ * step of Fig 4; "appended to the end of contig", left ends by symmetry P:L399-402).
+ * Extended contig c = ext(2c) + contig c + ext(2c+1), where ext(e) = ext_seq[ext_off[e]..ext_off[e+1])
+ * (LEFT extensions are already in contig-forward orientation, see la_result) — e.g. the ext_off /
+ * ext_seq that la_extend_device returns together with the batch's contig arrays.
+ * ALL pointers are device memory of the context's device; the call runs on the context stream and
+ * returns when the result is complete.  contig_off [n_contigs+1] and ext_off [2*n_contigs+1] are
+ * non-decreasing (their first elements need not be 0: offsets are taken relative to them).
+ * Outputs (caller-owned device memory): out_off [n_contigs+1], out_off[0] = 0, and out_seq of
+ * (contig_off[n]-contig_off[0]) + (ext_off[2n]-ext_off[0]) bytes.  The offsets are not validated
+ * on the device (inconsistent offsets are undefined behaviour).  Errors: LA_ERR_INVALID_ARG for
+ * n_contigs < 0 or NULL offset pointers, LA_ERR_CUDA (sticky) for a failed launch. */
+la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const char *contig_seq, const int64_t *contig_off,
+                               const int64_t *ext_off, const char *ext_seq, char *out_seq, int64_t *out_off);
 la_status la_get_stats(const la_ctx *ctx, la_stats *out);
 la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
 const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */

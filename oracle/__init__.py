@@ -100,3 +100,14 @@ def extend(batch, params, ends=None, loop_accepts=False):
     ext = [buf[i * W:i * W + int(ext_len[i])].decode() for i in range(n)]
     return dict(ends=ends, ext=ext, term=term, k_used=k_used, n_attempts=n_att, inserts=ins,
                 walk_steps=steps)
+
+
+def append_extensions(contigs, ext):
+    """Fig 4 "Append extensions to contigs" (L558-563) and P:L464 ("appended to the end of contig"),
+    both sides by the symmetry of P:L399-402: extended contig c = ext[2c] + contigs[c] + ext[2c+1],
+    ext[2c] (LEFT end) being in contig-forward orientation already (the oracle returns it so).
+    Plain definition, written out per contig."""
+    out = []
+    for c, seq in enumerate(contigs):
+        out.append(ext[2 * c] + seq + ext[2 * c + 1])
+    return out

@@ -53,8 +53,8 @@ class la_stats(ctypes.Structure):
                 ("prof_cycles", (ctypes.c_uint64 * 8) * 6)]
 
 
-EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_get_stats",
-           "la_destroy", "la_last_error", "la_plan_global_capacity", "la_paper_load_factor"]
+EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
+           "la_get_stats", "la_destroy", "la_last_error", "la_plan_global_capacity", "la_paper_load_factor"]
 
 _lib = None
 
@@ -81,6 +81,7 @@ def load():
     lib.la_extend_device.argtypes = [V, ctypes.POINTER(la_result)]
     lib.la_extend_streamed.argtypes = [V, ctypes.POINTER(la_batch), ctypes.POINTER(la_params), ctypes.c_int32,
                                        ctypes.POINTER(la_result)]
+    lib.la_append_extensions.argtypes = [V, ctypes.c_int32, V, V, V, V, V, V]
     lib.la_get_stats.argtypes = [V, ctypes.POINTER(la_stats)]
     lib.la_destroy.argtypes = [V]
     lib.la_last_error.argtypes = [V]
@@ -89,8 +90,8 @@ def load():
     lib.la_plan_global_capacity.restype = ctypes.c_int64
     lib.la_paper_load_factor.argtypes = [ctypes.c_int32, ctypes.c_int32]
     lib.la_paper_load_factor.restype = ctypes.c_double
-    for f in ("la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_get_stats",
-              "la_destroy"):
+    for f in ("la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
+              "la_get_stats", "la_destroy"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib

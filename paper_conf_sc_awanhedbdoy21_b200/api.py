@@ -136,6 +136,29 @@ class LocalAssembler:
         return dict(n_ends=int(r.n_ends), ext_off=r.ext_off, ext_seq=r.ext_seq, term=r.term,
                     k_used=r.k_used, n_attempts=r.n_attempts)
 
+    def append_extensions(self, contig_seq, contig_off, ext_off, ext_seq):
+        """la_append_extensions on CUDA tensors: extended contig c = ext(2c) + contig c + ext(2c+1)
+        (Fig 4 "Append extensions to contigs").  ext_off / ext_seq may be the
+        device pointers (ints) of extend_device() or CUDA tensors.  Returns (out_seq uint8, out_off
+        int64) CUDA tensors."""
+        import torch
+        n = int(contig_off.shape[0]) - 1
+        if not contig_off.is_cuda or not contig_seq.is_cuda:
+            raise ValueError("append_extensions: contig arrays must be CUDA tensors")
+        dev = contig_off.device
+        if isinstance(ext_off, int):   # extend_device() pointers: total length from la_get_stats
+            eoff_ptr, eseq_ptr = ext_off, ext_seq
+            ext_tot = int(self.stats()["ext_bases"])
+        else:
+            eoff_ptr, eseq_ptr = ext_off.data_ptr(), ext_seq.data_ptr()
+            ext_tot = int(ext_off[-1].item() - ext_off[0].item())
+        tot = int(contig_off[-1].item() - contig_off[0].item()) + ext_tot
+        out_seq = torch.empty(max(tot, 1), dtype=torch.uint8, device=dev)
+        out_off = torch.empty(n + 1, dtype=torch.int64, device=dev)
+        self._check(self._lib.la_append_extensions(self._ctx, n, contig_seq.data_ptr(), contig_off.data_ptr(),
+                                                   eoff_ptr, eseq_ptr, out_seq.data_ptr(), out_off.data_ptr()))
+        return out_seq[:tot], out_off
+
     def stats(self) -> dict:
         s = L.la_stats()
         self._check(self._lib.la_get_stats(self._ctx, ctypes.byref(s)))

@@ -1041,3 +1041,60 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
     return LA_OK;
 }
 extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, false); }
+
+// ---- NEXT N1: on-device append of extensions to contigs (Fig 4 "Append extensions to contigs",
+// P:L464 "appended to the end of contig") -------------------------------------------------------
+namespace la {
+// One warp per contig (grid-stride): out[c] = ext(2c) + contig c + ext(2c+1).  The output offset is
+// closed-form (no scan): out_off[c] = (contig_off[c] - contig_off[0]) + (ext_off[2c] - ext_off[0]),
+// because each contig's output is its two ends' extensions around it, in end order.  HBM-bound copy;
+// the byte loads/stores of a warp cover one 32-byte sector each, so the copy stays sector-efficient
+// for any alignment of the segments.
+__global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
+                                                    const int64_t *__restrict__ coff, const int64_t *__restrict__ eoff,
+                                                    const char *__restrict__ eseq, char *__restrict__ out,
+                                                    int64_t *__restrict__ out_off) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t c0 = coff[0], e0 = eoff[0];
+    for (int64_t c = warp0; c < n_contigs; c += nwarps) {
+        const int64_t cb = coff[c], ce = coff[c + 1];
+        const int64_t lb = eoff[2 * c], le = eoff[2 * c + 1], re = eoff[2 * c + 2];
+        const int64_t o = (cb - c0) + (lb - e0);
+        if (lane == 0) {
+            out_off[c] = o;
+            if (c == n_contigs - 1) out_off[n_contigs] = o + (ce - cb) + (re - lb);
+        }
+        char *dst = out + o;
+        for (int64_t i = lane; i < le - lb; i += 32) dst[i] = eseq[lb + i];
+        dst += le - lb;
+        for (int64_t i = lane; i < ce - cb; i += 32) dst[i] = cseq[cb + i];
+        dst += ce - cb;
+        for (int64_t i = lane; i < re - le; i += 32) dst[i] = eseq[le + i];
+    }
+}
+}  // namespace la
+
+extern "C" la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const char *contig_seq,
+                                          const int64_t *contig_off, const int64_t *ext_off, const char *ext_seq,
+                                          char *out_seq, int64_t *out_off) {
+    if (!ctx) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context is in a sticky CUDA error state");
+    if (n_contigs < 0 || !contig_off || !ext_off || !out_off)
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_append_extensions: n_contigs < 0 or a NULL offsets pointer");
+    CK(cudaSetDevice(ctx->device));
+    if (n_contigs == 0) {
+        CK(cudaMemsetAsync(out_off, 0, sizeof(int64_t), ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        return LA_OK;
+    }
+    const int threads = 256;
+    const int64_t want = ((int64_t)n_contigs * 32 + threads - 1) / threads;
+    const int blocks = (int)std::min<int64_t>(want, (int64_t)ctx->n_sm * 8);
+    k_append_ext<<<blocks, threads, 0, ctx->stream>>>(n_contigs, contig_seq, contig_off, ext_off, ext_seq, out_seq,
+                                                       out_off);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(ctx->stream));
+    return LA_OK;
+}

@@ -248,3 +248,44 @@ def test_assembler_k_rounds(LA, orc, k_start):
     for k", P:L150-160); k_start 77 starts on pointer (REF) keys, 55 upshifts into them."""
     b = cached_batch("C2", scale=0.03).select_contigs(np.arange(400))
     check(LA, orc, b, P0.replace(k_start=k_start, k_min=21, k_max=99))
+
+
+def _appended_strings(seq, off):
+    b = seq.cpu().numpy().tobytes()
+    o = off.cpu().numpy()
+    return [b[o[i]:o[i + 1]].decode() for i in range(o.shape[0] - 1)]
+
+
+def test_append_extensions_matches_oracle(LA, c2_ref):
+    """la_append_extensions (NEXT N1, Fig 4 "Append extensions to contigs"): device pipeline
+    load -> extend_device -> append, every extended contig equal to the oracle's
+    ext[2c] + contig + ext[2c+1]."""
+    import torch
+    import oracle
+    b, ref = c2_ref
+    contigs = [b.contig_seq[b.contig_off[c]:b.contig_off[c + 1]].tobytes().decode() for c in range(b.n_contigs)]
+    want = oracle.append_extensions(contigs, ref["ext"])
+    cseq = torch.from_numpy(b.contig_seq).cuda()
+    coff = torch.from_numpy(b.contig_off).cuda()
+    d = LA.load(b, P0).extend_device()
+    seq, off = LA.append_extensions(cseq, coff, d["ext_off"], d["ext_seq"])
+    assert int(off[0]) == 0 and int(off[-1]) == sum(len(x) for x in want)
+    assert _appended_strings(seq, off) == want
+
+
+def test_append_extensions_edge_cases(LA):
+    """Offsets not starting at 0 (a slice of a larger batch), empty extensions and contigs, none."""
+    import torch
+    import oracle
+    contigs = ["ACGTACGT", "", "GATTACA", "T"]
+    ext = ["CC", "", "A", "TTT", "", "", "G", "NACG"]
+    cseq = torch.tensor(list(b"XXXX" + "".join(contigs).encode()), dtype=torch.uint8).cuda()
+    coff = torch.tensor([4 + sum(len(x) for x in contigs[:i]) for i in range(5)], dtype=torch.int64).cuda()
+    eseq = torch.tensor(list(b"ZZ" + "".join(ext).encode()), dtype=torch.uint8).cuda()
+    eoff = torch.tensor([2 + sum(len(x) for x in ext[:i]) for i in range(9)], dtype=torch.int64).cuda()
+    seq, off = LA.append_extensions(cseq, coff, eoff, eseq)
+    assert _appended_strings(seq, off) == oracle.append_extensions(contigs, ext)
+    z = torch.zeros(1, dtype=torch.int64).cuda()
+    seq, off = LA.append_extensions(torch.zeros(0, dtype=torch.uint8).cuda(), z, z,
+                                    torch.zeros(0, dtype=torch.uint8).cuda())
+    assert seq.numel() == 0 and off.tolist() == [0]

@@ -308,3 +308,29 @@ def test_oracle_counters(orc):
     assert int(r["inserts"][0]) == len(reads) * ((150 - 33) + (150 - 25))
     n = p2_len(600, 150, 2, 500)
     assert int(r["walk_steps"][0]) == 2 * (n + 1)
+
+
+# ---- N1: append extensions to contigs (Fig 4) ---------------------------------
+def test_append_extensions_reassembles_genome(orc):
+    """An error-free contig G[500:700] with reads tiling both flanks: once both extensions are
+    appended, the extended contig is the contiguous genome window G[500-nl : 700+nr] — a left
+    extension prepended in the wrong orientation, or the ends swapped, breaks the window. The right
+    length is the P2 closed form."""
+    rng = np.random.default_rng(11)
+    G = C.unique_genome(rng, 1200)
+    l = 150
+    batch = C.single_end(G[500:700], C.tile(G, 560, 800, l), left_reads=C.tile(G, 300, 560, l))
+    r = orc.extend(batch, P0)
+    nl, nr = len(r["ext"][0]), len(r["ext"][1])
+    assert nr == p2_len(800, l, P0.min_votes, 700)
+    assert nl > 100
+    (out,) = orc.append_extensions([G[500:700]], r["ext"])
+    assert len(out) == nl + 200 + nr
+    assert out == G[500 - nl:700 + nr]
+
+
+def test_append_extensions_small():
+    import oracle
+    assert oracle.append_extensions(["ACGT", "", "GG"], ["TT", "CA", "", "", "A", ""]) == [
+        "TTACGTCA", "", "AGG"]
+    assert oracle.append_extensions([], []) == []
