@@ -1045,11 +1045,47 @@ extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return exte
 // ---- NEXT N1: on-device append of extensions to contigs (Fig 4 "Append extensions to contigs",
 // P:L464 "appended to the end of contig") -------------------------------------------------------
 namespace la {
+// Warp-cooperative copy of n bytes src -> dst for any alignment of either: byte copies up to the
+// first 16-byte-aligned destination address and after the last one, 16-byte stores in between.  Each
+// 16-byte destination chunk takes its source bytes from the two aligned 16-byte words that hold
+// them (both contain at least one byte of the source range, so they lie inside its allocation) and
+// realigns them with funnel shifts.  Every destination byte is written by exactly one lane.
+__device__ __forceinline__ void warp_copy(char *__restrict__ dst, const char *__restrict__ src, int64_t n, int lane) {
+    if (n <= 0) return;
+    const int64_t mis = (int64_t)((16 - ((uintptr_t)dst & 15)) & 15);
+    const int64_t head = n < mis ? n : mis;
+    if (lane < head) dst[lane] = src[lane];
+    const int64_t nbody = (n - head) >> 4;
+    const int64_t tail0 = head + (nbody << 4);
+    if (lane < n - tail0) dst[tail0 + lane] = src[tail0 + lane];
+    if (nbody == 0) return;
+    uint4 *__restrict__ d4 = reinterpret_cast<uint4 *>(dst + head);
+    const char *s = src + head;
+    const int sh = (int)((uintptr_t)s & 15);
+    const uint4 *__restrict__ s4 = reinterpret_cast<const uint4 *>(s - sh);
+    if (sh == 0) {
+        for (int64_t i = lane; i < nbody; i += 32) d4[i] = __ldg(s4 + i);
+        return;
+    }
+    const int q = sh >> 2, r = (sh & 3) * 8;
+    for (int64_t i = lane; i < nbody; i += 32) {
+        const uint4 lo = __ldg(s4 + i), hi = __ldg(s4 + i + 1);
+        const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+        uint32_t o[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const uint32_t a0 = q == 0 ? w[k] : q == 1 ? w[k + 1] : q == 2 ? w[k + 2] : w[k + 3];
+            const uint32_t a1 = q == 0 ? w[k + 1] : q == 1 ? w[k + 2] : q == 2 ? w[k + 3] : w[k + 4];
+            o[k] = __funnelshift_r(a0, a1, r);
+        }
+        d4[i] = make_uint4(o[0], o[1], o[2], o[3]);
+    }
+}
+
 // One warp per contig (grid-stride): out[c] = ext(2c) + contig c + ext(2c+1).  The output offset is
 // closed-form (no scan): out_off[c] = (contig_off[c] - contig_off[0]) + (ext_off[2c] - ext_off[0]),
-// because each contig's output is its two ends' extensions around it, in end order.  HBM-bound copy;
-// the byte loads/stores of a warp cover one 32-byte sector each, so the copy stays sector-efficient
-// for any alignment of the segments.
+// because each contig's output is its two ends' extensions around it, in end order.  HBM-bound copy
+// (algorithmic bytes: the sequence bytes read once and written once, plus the offsets).
 __global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
                                                     const int64_t *__restrict__ coff, const int64_t *__restrict__ eoff,
                                                     const char *__restrict__ eseq, char *__restrict__ out,
@@ -1067,11 +1103,11 @@ __global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const cha
             if (c == n_contigs - 1) out_off[n_contigs] = o + (ce - cb) + (re - lb);
         }
         char *dst = out + o;
-        for (int64_t i = lane; i < le - lb; i += 32) dst[i] = eseq[lb + i];
+        warp_copy(dst, eseq + lb, le - lb, lane);
         dst += le - lb;
-        for (int64_t i = lane; i < ce - cb; i += 32) dst[i] = cseq[cb + i];
+        warp_copy(dst, cseq + cb, ce - cb, lane);
         dst += ce - cb;
-        for (int64_t i = lane; i < re - le; i += 32) dst[i] = eseq[le + i];
+        warp_copy(dst, eseq + le, re - le, lane);
     }
 }
 }  // namespace la

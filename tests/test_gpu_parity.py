@@ -289,3 +289,25 @@ def test_append_extensions_edge_cases(LA):
     seq, off = LA.append_extensions(torch.zeros(0, dtype=torch.uint8).cuda(), z, z,
                                     torch.zeros(0, dtype=torch.uint8).cuda())
     assert seq.numel() == 0 and off.tolist() == [0]
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_append_extensions_alignments(LA, seed):
+    """Random segment lengths 0..300 and random leading offsets, so every source/destination
+    alignment (the 16-byte realigned copy, heads and tails) is exercised; against the oracle."""
+    import torch
+    import oracle
+    rng = np.random.default_rng(100 + seed)
+    n = 700
+
+    def rs(m):
+        return "".join(rng.choice(list("ACGTN"), m)) if m else ""
+    contigs = [rs(int(rng.integers(0, 300))) for _ in range(n)]
+    ext = [rs(int(rng.integers(0, 300)) if rng.random() < 0.8 else 0) for _ in range(2 * n)]
+    pc, pe = int(rng.integers(0, 16)), int(rng.integers(0, 16))
+    cseq = torch.tensor(list(b"x" * pc + "".join(contigs).encode()), dtype=torch.uint8).cuda()
+    eseq = torch.tensor(list(b"y" * pe + "".join(ext).encode()), dtype=torch.uint8).cuda()
+    coff = torch.from_numpy(pc + np.concatenate([[0], np.cumsum([len(x) for x in contigs])])).cuda()
+    eoff = torch.from_numpy(pe + np.concatenate([[0], np.cumsum([len(x) for x in ext])])).cuda()
+    seq, off = LA.append_extensions(cseq, coff, eoff, eseq)
+    assert _appended_strings(seq, off) == oracle.append_extensions(contigs, ext)
