@@ -1068,6 +1068,7 @@ __device__ __forceinline__ void warp_copy(char *__restrict__ dst, const char *__
         return;
     }
     const int q = sh >> 2, r = (sh & 3) * 8;
+#pragma unroll 2
     for (int64_t i = lane; i < nbody; i += 32) {
         const uint4 lo = __ldg(s4 + i), hi = __ldg(s4 + i + 1);
         const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
@@ -1086,7 +1087,7 @@ __device__ __forceinline__ void warp_copy(char *__restrict__ dst, const char *__
 // closed-form (no scan): out_off[c] = (contig_off[c] - contig_off[0]) + (ext_off[2c] - ext_off[0]),
 // because each contig's output is its two ends' extensions around it, in end order.  HBM-bound copy
 // (algorithmic bytes: the sequence bytes read once and written once, plus the offsets).
-__global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
+__global__ void __launch_bounds__(256, 4) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
                                                     const int64_t *__restrict__ coff, const int64_t *__restrict__ eoff,
                                                     const char *__restrict__ eseq, char *__restrict__ out,
                                                     int64_t *__restrict__ out_off) {
@@ -1094,9 +1095,20 @@ __global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const cha
     const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int64_t c0 = coff[0], e0 = eoff[0];
+    // the next contig's offsets are loaded before the current contig is copied (one offsets round
+    // trip per contig hidden behind the copy)
+    int64_t cb = 0, ce = 0, lb = 0, le = 0, re = 0;
+    if (warp0 < n_contigs) {
+        cb = coff[warp0], ce = coff[warp0 + 1];
+        lb = eoff[2 * warp0], le = eoff[2 * warp0 + 1], re = eoff[2 * warp0 + 2];
+    }
     for (int64_t c = warp0; c < n_contigs; c += nwarps) {
-        const int64_t cb = coff[c], ce = coff[c + 1];
-        const int64_t lb = eoff[2 * c], le = eoff[2 * c + 1], re = eoff[2 * c + 2];
+        const int64_t cn = c + nwarps;
+        int64_t ncb = 0, nce = 0, nlb = 0, nle = 0, nre = 0;
+        if (cn < n_contigs) {
+            ncb = coff[cn], nce = coff[cn + 1];
+            nlb = eoff[2 * cn], nle = eoff[2 * cn + 1], nre = eoff[2 * cn + 2];
+        }
         const int64_t o = (cb - c0) + (lb - e0);
         if (lane == 0) {
             out_off[c] = o;
@@ -1108,6 +1120,7 @@ __global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const cha
         warp_copy(dst, cseq + cb, ce - cb, lane);
         dst += ce - cb;
         warp_copy(dst, eseq + le, re - le, lane);
+        cb = ncb, ce = nce, lb = nlb, le = nle, re = nre;
     }
 }
 }  // namespace la
@@ -1127,7 +1140,9 @@ extern "C" la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const 
     }
     const int threads = 256;
     const int64_t want = ((int64_t)n_contigs * 32 + threads - 1) / threads;
-    const int blocks = (int)std::min<int64_t>(want, (int64_t)ctx->n_sm * 8);
+    int per_sm = 0;   // one full wave of resident CTAs (grid-stride over contigs)
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_append_ext, threads, 0));
+    const int blocks = (int)std::min<int64_t>(want, (int64_t)ctx->n_sm * std::max(per_sm, 1));
     k_append_ext<<<blocks, threads, 0, ctx->stream>>>(n_contigs, contig_seq, contig_off, ext_off, ext_seq, out_seq,
                                                        out_off);
     CK(cudaGetLastError());
