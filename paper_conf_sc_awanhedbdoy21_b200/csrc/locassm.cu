@@ -1045,44 +1045,63 @@ extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return exte
 // ---- NEXT N1: on-device append of extensions to contigs (Fig 4 "Append extensions to contigs",
 // P:L464 "appended to the end of contig") -------------------------------------------------------
 namespace la {
-// 16 source bytes starting at any address, from the two aligned 16-byte words that hold them (both
-// hold at least one byte of the requested range, so they lie inside its allocation), realigned with
-// funnel shifts.
-__device__ __forceinline__ uint4 load16_unaligned(const char *p) {
-    const int sh = (int)((uintptr_t)p & 15);
-    const uint4 *a = reinterpret_cast<const uint4 *>(p - sh);
-    const uint4 lo = __ldg(a);
-    if (sh == 0) return lo;
-    const uint4 hi = __ldg(a + 1);
-    const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
-    const int q = sh >> 2, r = (sh & 3) * 8;
-    uint32_t o[4];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        const uint32_t a0 = q == 0 ? w[k] : q == 1 ? w[k + 1] : q == 2 ? w[k + 2] : w[k + 3];
-        const uint32_t a1 = q == 0 ? w[k + 1] : q == 1 ? w[k + 2] : q == 2 ? w[k + 3] : w[k + 4];
-        o[k] = __funnelshift_r(a0, a1, r);
+// Warp-cooperative copy of n bytes src -> dst for any alignment of either: byte copies up to the
+// first 16-byte-aligned destination address and after the last one, 16-byte stores in between.  Each
+// 16-byte destination chunk takes its source bytes from the two aligned 16-byte words that hold
+// them (both contain at least one byte of the source range, so they lie inside its allocation) and
+// realigns them with funnel shifts.  Every destination byte is written by exactly one lane.
+__device__ __forceinline__ void warp_copy(char *__restrict__ dst, const char *__restrict__ src, int64_t n, int lane) {
+    if (n <= 0) return;
+    const int64_t mis = (int64_t)((16 - ((uintptr_t)dst & 15)) & 15);
+    const int64_t head = n < mis ? n : mis;
+    if (lane < head) dst[lane] = src[lane];
+    const int64_t nbody = (n - head) >> 4;
+    const int64_t tail0 = head + (nbody << 4);
+    if (lane < n - tail0) dst[tail0 + lane] = src[tail0 + lane];
+    if (nbody == 0) return;
+    uint4 *__restrict__ d4 = reinterpret_cast<uint4 *>(dst + head);
+    const char *s = src + head;
+    const int sh = (int)((uintptr_t)s & 15);
+    const uint4 *__restrict__ s4 = reinterpret_cast<const uint4 *>(s - sh);
+    if (sh == 0) {
+        for (int64_t i = lane; i < nbody; i += 32) d4[i] = __ldg(s4 + i);
+        return;
     }
-    return make_uint4(o[0], o[1], o[2], o[3]);
+    // lane i loads aligned source word i once; the following word comes from lane i+1 by shuffle
+    // (lane 31 loads it).  Word nbody is loaded only when sh != 0, where it holds the last chunk's
+    // final bytes.  The loop is warp-uniform, so the shuffles are convergent.
+    const int q = sh >> 2, r = (sh & 3) * 8;
+    for (int64_t i0 = 0; i0 < nbody; i0 += 32) {
+        const int64_t i = i0 + lane;
+        const uint4 z = make_uint4(0, 0, 0, 0);
+        const uint4 lo = i <= nbody ? __ldg(s4 + i) : z;
+        uint4 hi;
+        hi.x = __shfl_down_sync(0xffffffffu, lo.x, 1);
+        hi.y = __shfl_down_sync(0xffffffffu, lo.y, 1);
+        hi.z = __shfl_down_sync(0xffffffffu, lo.z, 1);
+        hi.w = __shfl_down_sync(0xffffffffu, lo.w, 1);
+        if (lane == 31) hi = i + 1 <= nbody ? __ldg(s4 + i + 1) : z;
+        if (i >= nbody) continue;
+        const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+        uint32_t o[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const uint32_t a0 = q == 0 ? w[k] : q == 1 ? w[k + 1] : q == 2 ? w[k + 2] : w[k + 3];
+            const uint32_t a1 = q == 0 ? w[k + 1] : q == 1 ? w[k + 2] : q == 2 ? w[k + 3] : w[k + 4];
+            o[k] = __funnelshift_r(a0, a1, r);
+        }
+        d4[i] = make_uint4(o[0], o[1], o[2], o[3]);
+    }
 }
 
 // One warp per contig (grid-stride): out[c] = ext(2c) + contig c + ext(2c+1).  The output offset is
 // closed-form (no scan): out_off[c] = (contig_off[c] - contig_off[0]) + (ext_off[2c] - ext_off[0]),
 // because each contig's output is its two ends' extensions around it, in end order.  HBM-bound copy
-// (algorithmic bytes: the sequence bytes read once and written once, plus the offsets).  The warp
-// treats the extended contig as one range of 16-byte-aligned output chunks, one chunk per lane: a
-// chunk inside one segment is one realigned 16-byte load, a chunk straddling a segment boundary
-// (at most two per contig) is gathered bytewise, and the unaligned head and tail of the range are
-// byte stores — so all of a contig's loads are in flight together.
-__device__ __forceinline__ char seg_byte(int64_t j, int64_t nl, int64_t nc, const char *l, const char *m,
-                                         const char *r) {
-    return j < nl ? l[j] : j < nl + nc ? m[j - nl] : r[j - nl - nc];
-}
-
-__global__ void __launch_bounds__(256, 5) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
-                                                       const int64_t *__restrict__ coff, const int64_t *__restrict__ eoff,
-                                                       const char *__restrict__ eseq, char *__restrict__ out,
-                                                       int64_t *__restrict__ out_off) {
+// (algorithmic bytes: the sequence bytes read once and written once, plus the offsets).
+__global__ void __launch_bounds__(256) k_append_ext(int64_t n_contigs, const char *__restrict__ cseq,
+                                                    const int64_t *__restrict__ coff, const int64_t *__restrict__ eoff,
+                                                    const char *__restrict__ eseq, char *__restrict__ out,
+                                                    int64_t *__restrict__ out_off) {
     const int lane = threadIdx.x & 31;
     const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -1091,43 +1110,16 @@ __global__ void __launch_bounds__(256, 5) k_append_ext(int64_t n_contigs, const 
         const int64_t cb = coff[c], ce = coff[c + 1];
         const int64_t lb = eoff[2 * c], le = eoff[2 * c + 1], re = eoff[2 * c + 2];
         const int64_t o = (cb - c0) + (lb - e0);
-        const int64_t nl = le - lb, nc = ce - cb, L = nl + nc + (re - le);
         if (lane == 0) {
             out_off[c] = o;
-            if (c == n_contigs - 1) out_off[n_contigs] = o + L;
+            if (c == n_contigs - 1) out_off[n_contigs] = o + (ce - cb) + (re - lb);
         }
-        const char *sl = eseq + lb, *sm = cseq + cb, *sr = eseq + le;
         char *dst = out + o;
-        const int64_t mis = (int64_t)((16 - ((uintptr_t)dst & 15)) & 15);
-        const int64_t head = L < mis ? L : mis;
-        const int64_t nbody = (L - head) >> 4;
-        const int64_t tail0 = head + (nbody << 4);
-        if (lane < head) dst[lane] = seg_byte(lane, nl, nc, sl, sm, sr);
-        if (lane < L - tail0) dst[tail0 + lane] = seg_byte(tail0 + lane, nl, nc, sl, sm, sr);
-        uint4 *__restrict__ d4 = reinterpret_cast<uint4 *>(dst + head);
-        for (int64_t i = lane; i < nbody; i += 32) {
-            const int64_t j = head + (i << 4);
-            uint4 v;
-            if (j + 16 <= nl) {
-                v = load16_unaligned(sl + j);
-            } else if (j >= nl && j + 16 <= nl + nc) {
-                v = load16_unaligned(sm + (j - nl));
-            } else if (j >= nl + nc) {
-                v = load16_unaligned(sr + (j - nl - nc));
-            } else {
-                uint32_t w[4];
-#pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    uint32_t x = 0;
-#pragma unroll
-                    for (int b = 0; b < 4; ++b)
-                        x |= (uint32_t)(uint8_t)seg_byte(j + 4 * k + b, nl, nc, sl, sm, sr) << (8 * b);
-                    w[k] = x;
-                }
-                v = make_uint4(w[0], w[1], w[2], w[3]);
-            }
-            d4[i] = v;
-        }
+        warp_copy(dst, eseq + lb, le - lb, lane);
+        dst += le - lb;
+        warp_copy(dst, cseq + cb, ce - cb, lane);
+        dst += ce - cb;
+        warp_copy(dst, eseq + le, re - le, lane);
     }
 }
 }  // namespace la
@@ -1147,9 +1139,7 @@ extern "C" la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const 
     }
     const int threads = 256;
     const int64_t want = ((int64_t)n_contigs * 32 + threads - 1) / threads;
-    int per_sm = 0;   // one full wave of resident CTAs (grid-stride over contigs)
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_append_ext, threads, 0));
-    const int blocks = (int)std::min<int64_t>(want, (int64_t)ctx->n_sm * std::max(per_sm, 1));
+    const int blocks = (int)std::min<int64_t>(want, (int64_t)ctx->n_sm * 8);
     k_append_ext<<<blocks, threads, 0, ctx->stream>>>(n_contigs, contig_seq, contig_off, ext_off, ext_seq, out_seq,
                                                        out_off);
     CK(cudaGetLastError());
