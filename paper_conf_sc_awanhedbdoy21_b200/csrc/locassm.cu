@@ -1067,21 +1067,9 @@ __device__ __forceinline__ void warp_copy(char *__restrict__ dst, const char *__
         for (int64_t i = lane; i < nbody; i += 32) d4[i] = __ldg(s4 + i);
         return;
     }
-    // lane i loads aligned source word i once; the following word comes from lane i+1 by shuffle
-    // (lane 31 loads it).  Word nbody is loaded only when sh != 0, where it holds the last chunk's
-    // final bytes.  The loop is warp-uniform, so the shuffles are convergent.
     const int q = sh >> 2, r = (sh & 3) * 8;
-    for (int64_t i0 = 0; i0 < nbody; i0 += 32) {
-        const int64_t i = i0 + lane;
-        const uint4 z = make_uint4(0, 0, 0, 0);
-        const uint4 lo = i <= nbody ? __ldg(s4 + i) : z;
-        uint4 hi;
-        hi.x = __shfl_down_sync(0xffffffffu, lo.x, 1);
-        hi.y = __shfl_down_sync(0xffffffffu, lo.y, 1);
-        hi.z = __shfl_down_sync(0xffffffffu, lo.z, 1);
-        hi.w = __shfl_down_sync(0xffffffffu, lo.w, 1);
-        if (lane == 31) hi = i + 1 <= nbody ? __ldg(s4 + i + 1) : z;
-        if (i >= nbody) continue;
+    for (int64_t i = lane; i < nbody; i += 32) {
+        const uint4 lo = __ldg(s4 + i), hi = __ldg(s4 + i + 1);
         const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
         uint32_t o[4];
 #pragma unroll
