@@ -57,3 +57,10 @@ def test_product_never_imports_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dp, f)).read()
                 assert "oracle" not in re.sub(r"#.*|//.*", "", txt).replace("oracle/", ""), f
+
+
+def test_append_extensions_null_context(lib):
+    """la_append_extensions rejects a NULL context without touching the device."""
+    lib.la_append_extensions.argtypes = [ctypes.c_void_p, ctypes.c_int32] + [ctypes.c_void_p] * 6
+    lib.la_append_extensions.restype = ctypes.c_int
+    assert lib.la_append_extensions(None, 0, None, None, None, None, None, None) == -1
