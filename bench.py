@@ -320,6 +320,25 @@ def main():
     ms_smem = statistics.mean(s["ms_smem"] for s in stats)
     launches = sum(s["kernel_launches"] for s in stats)
 
+    # ---------------- NEXT N1: on-device append of the extensions (not part of the step) ----------------
+    d = la.extend_device()
+    ap_ms = []
+    for i in range(6):
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        la.append_extensions(dev.contig_seq, dev.contig_off, d["ext_off"], d["ext_seq"])
+        a1.record(stream)
+        a1.synchronize()
+        if i:
+            ap_ms.append(a0.elapsed_time(a1))
+    ap_bytes = 2 * (int(batch.contig_off[-1] - batch.contig_off[0]) + int(la.stats()["ext_bases"])) + \
+        8 * (4 * batch.n_contigs + 3)
+    ap_med = statistics.median(ap_ms)
+    append_n1 = {"kernel": "k_append_ext", "ms": ap_med, "bound": "hbm", "algorithmic_bytes": ap_bytes,
+                 "achieved": ap_bytes / (ap_med / 1e3) / 1e9, "unit": "GB/s",
+                 "note": "la_append_extensions on this step's results, CUDA events around the call (includes "
+                         "its launch); outside the timed step; DESIGN.md §10a"}
+
     # ---------------- end to end through the public API (host buffers) ----------------
     e2e = None
     if not args.no_e2e:
@@ -422,6 +441,7 @@ def main():
         "clocks": clk.summary(),
         "e2e": e2e,
         "gather_ms": gather_ms,
+        "append_n1": dict(append_n1, peak=peaks["hbm_gbs"], frac=append_n1["achieved"] / peaks["hbm_gbs"]),
     }
     if not args.no_cpu_baseline and world == 1:
         v, eps, cores, desc = cpu_oracle_sample(batch, params, budget_s=args.ref_budget)
