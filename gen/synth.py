@@ -21,6 +21,7 @@ from .batch import Batch, _ranges_to_ids
 
 ASCII = np.frombuffer(b"ACGTN", np.uint8)
 RL = 150                      # read length (150 bp reads)
+GEN_VERSION = 2               # bumped when a config's recipe changes (bench.py cache key)
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libsynth.so")
@@ -368,7 +369,7 @@ def c3_cfg(seed: int = seed_for(2)) -> MetaCfg:
     return MetaCfg("C3", sp, n_me_fam=10)
 
 
-def c4_cfg(seed: int = seed_for(3), scale: float = 1.0) -> MetaCfg:
+def c4_cfg(seed: int = seed_for(3), scale: float = 1.0, cut_rate: float = 1 / 400) -> MetaCfg:
     """Paper-shaped: 500 species 0.5-6 Mbp (~1.1 Gbp), lognormal(0,1.5) abundance, ~100M reads."""
     rng = np.random.default_rng(seed ^ 0x5EED)
     n = max(2, int(round(500 * scale)))
@@ -377,7 +378,9 @@ def c4_cfg(seed: int = seed_for(3), scale: float = 1.0) -> MetaCfg:
     a = rng.lognormal(0.0, 1.5, n)
     total_reads = 100e6 * scale
     cov = a * total_reads * RL / float((a * L).sum())
-    sp = [Species(int(L[i]), float(gc[i]), float(cov[i]), cut_rate=1 / 2000) for i in range(n)]
+    # breakpoint rate tuned so the batch has ~1M contigs (2M ends), the size SURVEY §8(d) states for
+    # C4 (r01 used 1/2000: 510k contigs); ~97M candidate-read copies
+    sp = [Species(int(L[i]), float(gc[i]), float(cov[i]), cut_rate=cut_rate) for i in range(n)]
     return MetaCfg("C4", sp)
 
 
@@ -395,4 +398,7 @@ def make(config: str, seed: int | None = None, **kw) -> Batch:
     if config in ("C4", "C5"):
         s = seed if seed is not None else seed_for(3)
         return make_metagenome(c4_cfg(s, kw.pop("scale", 1.0)), s, **kw)
+    if config == "C4S":   # r01's C4 (510k contigs, 31.7M read copies): quicker A/B comparisons
+        s = seed if seed is not None else seed_for(3)
+        return make_metagenome(c4_cfg(s, kw.pop("scale", 1.0), cut_rate=1 / 2000), s, **kw)
     raise ValueError(f"unknown config {config}")

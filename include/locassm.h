@@ -51,6 +51,8 @@ typedef enum {
 
 typedef enum { LA_MEM_HOST = 0, LA_MEM_DEVICE = 1 } la_mem;
 
+#define LA_HIST 16
+
 typedef struct {
     int32_t k_start, k_min, k_max, k_shift; /* 1 <= k_min <= k_start <= k_max <= 128; k_shift >= 1 */
     int32_t max_walk_len;                   /* W: 0 <= W <= 1024 (paper: walks up to 300) */
@@ -117,6 +119,15 @@ typedef struct {
     /* LA_PROFILE=1 only: per class, summed clock64 cycles of the builders' leader (wait for the
        walker, prefix, clear, filter pass, build pass, link) and of the walker (wait, walk) */
     uint64_t prof_cycles[6][8];
+    /* hash-build / walk split (SURVEY.md §8(b), §8(d) timing step 5), set by la_replay_build
+       (-1 until then): ms_build = device time of the build-only replay of the table-class kernels,
+       ms_walk = ms_smem - ms_build (link pass, walk and hand-offs); per class likewise */
+    double ms_build, ms_walk;
+    double cls_build_ms[6];
+    int64_t cls_build_inserts[6];
+    /* per class: attempts built with inline keys (k <= 63) and with pointer keys (k >= 64) */
+    int64_t cls_inl_attempts[6], cls_ref_attempts[6];
+    int64_t attempts_hist[LA_HIST]; /* ends by number of attempts (last bin: >= LA_HIST-1)       */
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);
@@ -153,6 +164,14 @@ la_status la_extend_streamed(la_ctx *ctx, const la_batch *batch, const la_params
  * n_contigs < 0 or NULL offset pointers, LA_ERR_CUDA (sticky) for a failed launch. */
 la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const char *contig_seq, const int64_t *contig_off,
                                const int64_t *ext_off, const char *ext_seq, char *out_seq, int64_t *out_off);
+/* Build-only replay of the last la_extend (SURVEY.md §8(d) timing protocol step 5, "the hash-build
+ * phase"): reruns, on the device, exactly the (end, k) table builds that la_extend made in its
+ * shared-memory / XL table classes — read staging, per-read prefix, table clear, filter and build
+ * passes of Alg 1 — with the link pass and the walk disabled, and records the device
+ * time in la_stats.ms_build / cls_build_ms and the replayed inserts in cls_build_inserts.  Results
+ * of the last la_extend are unchanged.  Errors: LA_ERR_STATE if no la_extend completed since the
+ * last la_load_batch; LA_ERR_CUDA (sticky). */
+la_status la_replay_build(la_ctx *ctx);
 la_status la_get_stats(const la_ctx *ctx, la_stats *out);
 la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
 const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */

@@ -13,6 +13,7 @@ SO = os.environ.get("LA_SO") or os.path.join(HERE, "liblocassm.so")   # LA_SO: d
 
 LA_OK, LA_ERR_INVALID_ARG, LA_ERR_OOM, LA_ERR_CUDA, LA_ERR_STATE, LA_ERR_CAPACITY = 0, -1, -2, -3, -4, -5
 LA_MEM_HOST, LA_MEM_DEVICE = 0, 1
+LA_HIST = 16
 STATUS = {0: "LA_OK", -1: "LA_ERR_INVALID_ARG", -2: "LA_ERR_OOM", -3: "LA_ERR_CUDA",
           -4: "LA_ERR_STATE", -5: "LA_ERR_CAPACITY"}
 TERM_NAMES = ["DEADEND", "FORK", "LOOP", "MAXLEN", "NOREADS", "SHORT"]
@@ -50,10 +51,15 @@ class la_stats(ctypes.Structure):
                 ("xl_scratch_bytes", ctypes.c_int64), ("cls_ends", ctypes.c_int64 * 6),
                 ("cls_inserts", ctypes.c_int64 * 6), ("cls_attempts", ctypes.c_int64 * 6),
                 ("cls_filtered", ctypes.c_int64 * 6), ("cls_ms", ctypes.c_double * 6),
-                ("prof_cycles", (ctypes.c_uint64 * 8) * 6)]
+                ("prof_cycles", (ctypes.c_uint64 * 8) * 6),
+                ("ms_build", ctypes.c_double), ("ms_walk", ctypes.c_double),
+                ("cls_build_ms", ctypes.c_double * 6), ("cls_build_inserts", ctypes.c_int64 * 6),
+                ("cls_inl_attempts", ctypes.c_int64 * 6), ("cls_ref_attempts", ctypes.c_int64 * 6),
+                ("attempts_hist", ctypes.c_int64 * LA_HIST)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
+           "la_replay_build",
            "la_get_stats", "la_destroy", "la_last_error", "la_plan_global_capacity", "la_paper_load_factor"]
 
 _lib = None
@@ -83,6 +89,7 @@ def load():
                                        ctypes.POINTER(la_result)]
     lib.la_append_extensions.argtypes = [V, ctypes.c_int32, V, V, V, V, V, V]
     lib.la_get_stats.argtypes = [V, ctypes.POINTER(la_stats)]
+    lib.la_replay_build.argtypes = [V]
     lib.la_destroy.argtypes = [V]
     lib.la_last_error.argtypes = [V]
     lib.la_last_error.restype = ctypes.c_char_p
@@ -91,7 +98,7 @@ def load():
     lib.la_paper_load_factor.argtypes = [ctypes.c_int32, ctypes.c_int32]
     lib.la_paper_load_factor.restype = ctypes.c_double
     for f in ("la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
-              "la_get_stats", "la_destroy"):
+              "la_replay_build", "la_get_stats", "la_destroy"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib

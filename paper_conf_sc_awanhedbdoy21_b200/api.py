@@ -27,15 +27,31 @@ def _params(p) -> L.la_params:
     return L.la_params(*[int(get(n)) for n in PARAM_FIELDS])
 
 
-def _ptr_and_mem(a):
-    """(pointer, is_device, keepalive) of a numpy array or torch tensor."""
+_BYTE_KINDS = ("uint8", "int8")
+
+
+def _ptr_and_mem(a, name, want, device=None):
+    """(pointer, is_device, keepalive) of a numpy array or torch tensor.  The library reads offsets as
+    int64 and sequences as bytes: any other dtype (e.g. int32 offsets from a cumsum), a tensor on
+    another GPU than the context's, or a non-contiguous layout is rejected here (ValueError)
+    instead of being read out of bounds in C."""
     try:
         import torch
         if isinstance(a, torch.Tensor):
+            dt = str(a.dtype).replace("torch.", "")
+            if (want == "int64" and dt != "int64") or (want == "bytes" and dt not in _BYTE_KINDS):
+                raise ValueError(f"{name}: dtype {dt}, need {'int64' if want == 'int64' else 'uint8/int8'}")
+            if a.is_cuda and device is not None and a.device.index != device:
+                raise ValueError(f"{name}: tensor on cuda:{a.device.index}, the context is on cuda:{device}")
             a = a.contiguous()
             return a.data_ptr(), a.is_cuda, a
     except ImportError:  # pragma: no cover
         pass
+    a = np.asarray(a)
+    if want == "int64" and a.dtype != np.int64:
+        raise ValueError(f"{name}: dtype {a.dtype}, need int64")
+    if want == "bytes" and a.dtype not in (np.uint8, np.int8):
+        raise ValueError(f"{name}: dtype {a.dtype}, need uint8/int8")
     a = np.ascontiguousarray(a)
     return a.ctypes.data, False, a
 
@@ -74,20 +90,24 @@ class LocalAssembler:
         if st != L.LA_OK:
             raise L.LocAssmError(st, "la_create failed (no CUDA device?)")
         self._keep = None
+        self._device = int(device)
 
     def _check(self, st):
         if st != L.LA_OK:
             raise L.LocAssmError(st, self._lib.la_last_error(self._ctx).decode())
 
-    @staticmethod
-    def _batch(batch):
-        arrs = [batch.contig_seq, batch.contig_off, batch.read_seq, batch.read_qual, batch.read_off,
-                batch.end_read_off]
-        ptrs, devs, keep = zip(*[_ptr_and_mem(a) for a in arrs])
+    _FIELDS = (("contig_seq", "bytes"), ("contig_off", "int64"), ("read_seq", "bytes"), ("read_qual", "bytes"),
+               ("read_off", "int64"), ("end_read_off", "int64"))
+
+    def _batch(self, batch):
+        arrs = [getattr(batch, f) for f, _ in self._FIELDS]
+        ptrs, devs, keep = zip(*[_ptr_and_mem(a, f, w, self._device) for a, (f, w) in zip(arrs, self._FIELDS)])
         if len(set(devs)) != 1:
             raise ValueError("batch arrays must all be host or all be device memory")
         n_contigs = int(arrs[1].shape[0]) - 1
         n_reads = int(arrs[4].shape[0]) - 1
+        if 2 * n_contigs + 1 != int(arrs[5].shape[0]):
+            raise ValueError("end_read_off must have 2*n_contigs+1 entries")
         b = L.la_batch(L.LA_MEM_DEVICE if devs[0] else L.LA_MEM_HOST, n_contigs, ptrs[0], ptrs[1], n_reads,
                        ptrs[2], ptrs[3], ptrs[4], ptrs[5])
         return b, keep
@@ -145,6 +165,15 @@ class LocalAssembler:
         n = int(contig_off.shape[0]) - 1
         if not contig_off.is_cuda or not contig_seq.is_cuda:
             raise ValueError("append_extensions: contig arrays must be CUDA tensors")
+        for name, t, ok in (("contig_off", contig_off, (torch.int64,)), ("contig_seq", contig_seq, (torch.uint8, torch.int8))) + (
+                () if isinstance(ext_off, int) else
+                (("ext_off", ext_off, (torch.int64,)), ("ext_seq", ext_seq, (torch.uint8, torch.int8)))):
+            if t.dtype not in ok:
+                raise ValueError(f"append_extensions: {name} has dtype {t.dtype}")
+            if not t.is_cuda or t.device.index != self._device:
+                raise ValueError(f"append_extensions: {name} must be a CUDA tensor on cuda:{self._device}")
+            if not t.is_contiguous():
+                raise ValueError(f"append_extensions: {name} must be contiguous")
         dev = contig_off.device
         if isinstance(ext_off, int):   # extend_device() pointers: total length from la_get_stats
             eoff_ptr, eseq_ptr = ext_off, ext_seq
@@ -158,6 +187,12 @@ class LocalAssembler:
         self._check(self._lib.la_append_extensions(self._ctx, n, contig_seq.data_ptr(), contig_off.data_ptr(),
                                                    eoff_ptr, eseq_ptr, out_seq.data_ptr(), out_off.data_ptr()))
         return out_seq[:tot], out_off
+
+    def replay_build(self) -> dict:
+        """la_replay_build: rerun the last extension's table builds only (the hash-build phase) and
+        return the stats with ms_build / cls_build_ms / cls_build_inserts filled in."""
+        self._check(self._lib.la_replay_build(self._ctx))
+        return self.stats()
 
     def stats(self) -> dict:
         s = L.la_stats()

@@ -64,52 +64,11 @@ __global__ void k_read_end(const int64_t *__restrict__ eoff, int64_t n_ends, int
     read_end[j] = (int32_t)lo;
 }
 
-// one thread per (read, 32-base word): oriented 2-bit bases and quality classes.
-// LEFT-end reads are reverse complemented with reversed qualities (reading #14).
-__global__ void k_encode_reads(const char *__restrict__ seq, const char *__restrict__ qual,
-                               const int64_t *__restrict__ roff, const int32_t *__restrict__ read_end,
-                               int64_t n_reads, int SW, DevParams P, uint64_t *__restrict__ rseq,
-                               uint64_t *__restrict__ rqc, uint16_t *__restrict__ rlen,
-                               uint8_t *__restrict__ rflag, uint32_t *err) {
-    int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    int64_t j = t / SW;
-    int w = (int)(t - j * SW);
-    if (j >= n_reads) return;
-    const int64_t o = roff[j];
-    const int len = (int)(roff[j + 1] - o);
-    const bool left = (read_end[j] & 1) == 0;
-    uint64_t sb = 0, qb = 0;
-    uint32_t e = 0;
-    bool hasN = false;
-    for (int i = 0; i < 32; ++i) {
-        int ib = w * 32 + i;
-        uint32_t code = 0, qc = 0;
-        if (ib < len) {
-            int64_t src = left ? o + len - 1 - ib : o + ib;
-            int c = base_code((unsigned char)seq[src]);
-            int q = (int)(unsigned char)qual[src] - P.qual_offset;
-            if (c < 0) { e |= ERR_READ_CHAR; c = 4; }
-            if (q < 0) e |= ERR_QUAL_CHAR;
-            if (c == 4) { code = 0; qc = 3; hasN = true; }
-            else {
-                code = left ? 3 - c : c;
-                qc = q >= P.q_hi ? 2 : (q >= P.q_lo ? 1 : 0);
-            }
-        }
-        sb |= (uint64_t)code << (62 - 2 * i);
-        qb |= (uint64_t)qc << (62 - 2 * i);
-    }
-    rseq[j * SW + w] = sb;
-    rqc[j * SW + w] = qb;
-    if (e) atomicOr(err, e);
-    if (w == 0) rlen[j] = (uint16_t)len;
-    if (hasN) rflag[j] = 1;   // rflag zeroed before launch
-}
-
-// Staged variant (the one la_load_batch launches): a CTA takes ENC_R consecutive reads, copies their
-// contiguous byte range of seq and qual into shared memory with coalesced 16 B loads, then one thread
-// per (read, 32-base word) packs from shared memory.  The per-thread global byte loads of
-// k_encode_reads ran at ~0.45 TB/s on C4 (ncu r01); this streams the ASCII input once, coalesced.
+// Read encoder (a2): oriented 2-bit bases and quality classes; LEFT-end reads are reverse
+// complemented with reversed qualities (reading #14).  A CTA takes ENC_R consecutive
+// reads, copies their contiguous byte range of seq and qual into shared memory with coalesced 16 B
+// loads, then one thread per (read, 32-base word) packs from shared memory (r01: a thread-per-word
+// encoder doing per-thread global byte loads ran at ~0.45 TB/s on C4 and was removed).
 constexpr int ENC_R = 64;
 constexpr int ENC_BYTES = ENC_R * MAX_READ_LEN + 32;
 __global__ void __launch_bounds__(256) k_encode_reads_staged(
@@ -243,6 +202,17 @@ namespace la {
 // ------------------------------------------------------------------------------------------------
 // emit (a9)
 // ------------------------------------------------------------------------------------------------
+// ends per attempt count (la_stats.attempts_hist; the last bin collects >= LA_HIST - 1)
+__global__ void k_att_hist(const uint8_t *__restrict__ att, int64_t n, unsigned long long *__restrict__ hist) {
+    __shared__ unsigned int h[LA_HIST];
+    if (threadIdx.x < LA_HIST) h[threadIdx.x] = 0;
+    __syncthreads();
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) atomicAdd(&h[min((int)att[i], LA_HIST - 1)], 1u);
+    __syncthreads();
+    if (threadIdx.x < LA_HIST && h[threadIdx.x]) atomicAdd(&hist[threadIdx.x], (unsigned long long)h[threadIdx.x]);
+}
+
 __global__ void k_len64(const int32_t *__restrict__ len, int64_t n, int64_t *__restrict__ out) {
     int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i < n) out[i] = len[i];

@@ -23,6 +23,8 @@
 //           the walk of one end overlaps the build of the other; XL streams reads from L2/HBM.
 #pragma once
 #include "la_device.cuh"
+#include "la_inl32.cuh"
+#include <type_traits>
 
 namespace la {
 
@@ -40,6 +42,9 @@ __device__ __forceinline__ long long la_clock() {
 #endif
 }
 
+#ifndef LA_FQUEUE
+#define LA_FQUEUE 0   // 1: filtered builds keep per-position filter indices and queue survivors (r02 experiment)
+#endif
 #ifndef LA_MAX_LOAD
 #define LA_MAX_LOAD 0.70f
 #endif
@@ -55,16 +60,22 @@ struct SmemFixed {
     uint32_t icap;        // slots an info buffer can describe (max table capacity)
     uint32_t off_info1, off_walk, off_tab, tab_bytes;
     uint32_t off_filt, filt_bytes;   // XL only: the filter bitmaps stay in shared memory
+    uint32_t off_queue;              // per builder warp: 64 x u32 survivor queue (build pass)
 };
+// survivor queue of the build pass (la_inl32.cuh): 64 positions per builder warp
+__host__ __device__ __forceinline__ uint32_t queue_bytes(int nbw) { return LA_FQUEUE ? (uint32_t)nbw * 64u * 4u : 0u; }
 
 constexpr uint32_t XL_ICAP = 16384u;   // XL: info buffers of 64 KB each; the rest of smem = filter
 
 // gt_stride > 0: the table lives in a per-CTA global-memory scratch of gt_stride bytes (XL class);
 // shared memory then holds the two info buffers, the walk strings and the filter bitmaps.
 // single = true: one end in flight (k_small): one info buffer and two walk strings.
-__host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, uint32_t gt_stride = 0,
-                                                         bool single = false) {
+__host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, uint32_t gt_stride, bool single,
+                                                         int nbw) {
     SmemFixed F;
+    const uint32_t qb = queue_bytes(nbw);   // the queues sit at the end of the dynamic region
+    bytes = bytes > qb + 256u ? ((bytes - qb) & ~15u) : 0u;
+    F.off_queue = bytes;
     const uint32_t Wp = ((uint32_t)W + 15u) & ~15u;
     const uint32_t nwalk = single ? 2u : 4u;
     const uint32_t fixed = nwalk * Wp + 128u;
@@ -95,6 +106,7 @@ __host__ __device__ __forceinline__ SmemFixed smem_fixed(int W, uint32_t bytes, 
 
 struct SmemTab {
     uint32_t off_pref, off_b1, off_b2, off_keys, off_cnts, off_list, cap, mwords;
+    uint32_t off_f;   // filtered tables: per position its filter bit index (u16 shared / u32 XL global)
 };
 
 __host__ __device__ __forceinline__ uint32_t pref_bytes(int r) { return (((uint32_t)r + 1u) * 4u + 15u) & ~15u; }
@@ -102,6 +114,12 @@ __host__ __device__ __forceinline__ uint32_t pref_bytes(int r) { return (((uint3
 // u8 has-N flag
 __host__ __device__ __forceinline__ uint32_t stage_bytes(int r, int SW) {
     return (((uint32_t)r * (uint32_t)SW * 16u + (uint32_t)r * 3u) + 15u) & ~15u;
+}
+// per-position filter indices of a filtered build (la_inl32.cuh): u16 in shared memory (bit indices
+// < 65535, so at most MAX_SMEM_MBITS filter bits), u32 in the XL class's global scratch
+constexpr uint32_t MAX_SMEM_MBITS = 65504u;
+__host__ __device__ __forceinline__ uint32_t fpos_bytes(uint32_t U, bool gt) {
+    return LA_FQUEUE ? (((gt ? 4u : 2u) * U + 15u) & ~15u) : 0u;
 }
 
 // U = voting-occurrence upper bound (sum over reads of max(0, len-k)); the table region starts with
@@ -135,12 +153,15 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
         T.off_keys = pb;
     } else {
         if (filt) {
-            // two bitmaps of ~4 bits per occurrence each, at most a quarter of the region each
+            // two bitmaps of ~4 bits per occurrence each (at most a quarter of the region each and
+            // MAX_SMEM_MBITS bits), then the u16 filter index of every position
             mwords = (4u * U + 31u) / 32u;
             const uint32_t maxw = tab / 16u;
             if (mwords > maxw) mwords = maxw;
-            mwords = (mwords + 3u) & ~3u;
-            const uint32_t rem = tab > 8u * mwords + 16u ? tab - 8u * mwords - 16u : 0u;
+            if (LA_FQUEUE && mwords > MAX_SMEM_MBITS / 32u) mwords = MAX_SMEM_MBITS / 32u;
+            mwords &= ~3u;
+            const uint32_t used = 8u * mwords + fpos_bytes(U, false) + 16u;
+            const uint32_t rem = tab > used ? tab - used : 0u;
             cap = rem / per_slot;
             if (cap > F.icap) cap = F.icap;
             cap &= ~1u;
@@ -148,12 +169,14 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
         T.off_pref = F.off_tab + sb;
         T.off_b1 = F.off_tab + pb;
         T.off_b2 = T.off_b1 + mwords * 4u;
-        T.off_keys = (T.off_b2 + mwords * 4u + 15u) & ~15u;
+        T.off_keys = (T.off_b2 + mwords * 4u + (mwords ? fpos_bytes(U, false) : 0u) + 15u) & ~15u;
     }
     T.cap = cap;
     T.mwords = mwords;
     T.off_cnts = T.off_keys + cap * kbytes;
     T.off_list = T.off_cnts + cap * cnt_bytes(gt);
+    // shared: right after B2; XL: in the global scratch after the claim list
+    T.off_f = gt ? ((T.off_list + cap * 2u + 15u) & ~15u) : (T.off_b2 + mwords * 4u);
     return T;
 }
 
@@ -165,10 +188,13 @@ __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
     return r < 50 ? 0.30f : (r < 200 ? 0.16f : 0.10f);
 }
 
-__device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t min_cap,
+__host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { return 4u * threads; }
+
+__device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t threads,
                                      int SW, bool single) {
+    const uint32_t min_cap = min_table_cap(threads);
     if (bytes == 0) return false;
-    const SmemFixed F = smem_fixed(P.W, bytes, 0u, single);
+    const SmemFixed F = smem_fixed(P.W, bytes, 0u, single, single ? (int)(threads / 32u) : (int)(threads / 32u) - 1);
     if (F.tab_bytes == 0) return false;
     if (r > 16384) return false;
     const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r, false, SW);
@@ -187,7 +213,6 @@ struct PlanBytes {
     uint32_t single;              // bit i: class i runs k_small (one end per CTA, no walker warp)
 };
 
-__host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { return 4u * threads; }
 
 // XL class: 512-thread CTAs (1 per SM) whose tables live in a per-CTA global-memory scratch (L2-resident
 // for the paper-shaped batch); shared memory keeps the info buffers (so the walk stays on-chip).
@@ -205,12 +230,13 @@ __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_
     uint32_t cap = xl_needed_cap(r_max, U_max, filter);
     if (cap < min_table_cap(XL_THREADS)) cap = min_table_cap(XL_THREADS);   // claims + in-flight < cap
     if (cap > icap) cap = icap;
-    return (pref_bytes((int)r_max) + 32u + cap * (16u + cnt_bytes(true) + 2u) + 255u) & ~255u;
+    return (pref_bytes((int)r_max) + 48u + cap * (16u + cnt_bytes(true) + 2u) + fpos_bytes((uint32_t)U_max, true) +
+            255u) & ~255u;
 }
 
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
                        const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW, PlanBytes pb,
-                       uint32_t xl_bytes,
+                       uint32_t xl_bytes, int force_cls,
                        int32_t *__restrict__ cls, int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
                        uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att, int32_t *__restrict__ lists,
                        uint32_t *__restrict__ keys, int32_t *__restrict__ list_G, int *__restrict__ ctr) {
@@ -222,19 +248,26 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
     if (r == 0) c = CLS_NOREADS;
     else if (clen[e] < P.k_start) c = CLS_SHORT;
     else {
-        const int64_t sumlen = roff[eoff[e + 1]] - roff[eoff[e]];
-        int64_t U = sumlen - r * (int64_t)P.k_min;   // occurrences at the smallest k of the schedule
-        if (U < 0) U = 0;
+        // exact voting-occurrence bounds U(k) = sum over reads of max(0, len - k) at the smallest k of
+        // the schedule (table sizing) and at k_start (LPT key); reads shorter than k contribute 0
+        int64_t U = 0, U0 = 0;
+        for (int64_t j = eoff[e]; j < eoff[e + 1]; ++j) {
+            const int64_t l = roff[j + 1] - roff[j];
+            U += l > P.k_min ? l - P.k_min : 0;
+            U0 += l > P.k_start ? l - P.k_start : 0;
+        }
         c = CLS_GLOBAL;
         int sc = -1;
         if (U < (1ll << 30))
             for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
-                if (fits(r, U, P, pb.b[i], min_table_cap(pb.t[i]), SW, (pb.single >> i) & 1u)) sc = i;
-        int64_t U0 = sumlen - r * (int64_t)P.k_start;   // LPT key: occurrences at k_start
-        U0 = U0 < 0 ? 0 : (U0 > 0xffffffffll ? 0xffffffffll : U0);
+                if (fits(r, U, P, pb.b[i], pb.t[i], SW, (pb.single >> i) & 1u)) sc = i;
+        U0 = U0 > 0xffffffffll ? 0xffffffffll : U0;
         if (sc < 0 && xl_bytes && r <= 16384 && U <= XL_MAX_U &&
-            xl_needed_cap(r, U, P.V >= 2) <= smem_fixed(P.W, xl_bytes, 1u).icap)
+            xl_needed_cap(r, U, P.V >= 2) <= smem_fixed(P.W, xl_bytes, 1u, false, XL_THREADS / 32 - 1).icap)
             sc = N_SMEM_CLASSES;   // XL: table in global scratch
+        // test hook (LA_FORCE_CLASS): every end with reads in one class; ends whose table does not
+        // fit there overflow and are redone by the global path
+        if (force_cls >= 0 && r <= 16384 && U <= XL_MAX_U) sc = force_cls;
         if (sc >= 0) {
             c = CLS_S + sc;
             const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : sc], 1);
@@ -262,8 +295,15 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
 constexpr uint32_t NEXT_NONE = 0x0FFFFFFFu;   // info word: next slot (28 bits) << 4 | visited << 3 | code
 
 struct GlobalStats {
-    unsigned long long inserts, steps, attempts, filtered;   // filtered: attempts built with the filter
+    // filtered: attempts built with the filter; inl / ref: attempts with inline / pointer (REF) keys
+    unsigned long long inserts, steps, attempts, filtered, inl, ref;
 };
+constexpr int GSTATS_WORDS = 6;
+// out_dir[e]: direction of the end's k shifts (-1 down, +1 up, 0 none) recorded by the extension,
+// so that la_replay_build can rerun exactly the same (end, k) attempts; OVF_DIR: the end left the
+// class kernel (table overflow -> global path) and is not replayed.
+constexpr int8_t OVF_DIR = 127;
+__device__ __forceinline__ int8_t shift_dir(int shift) { return (int8_t)(shift > 0 ? 1 : (shift < 0 ? -1 : 0)); }
 
 __device__ __forceinline__ uint32_t filt_index(uint64_t h, uint32_t mbits) {
     return (uint32_t)(((h >> 32) * (uint64_t)mbits) >> 32);
@@ -301,14 +341,6 @@ __device__ __forceinline__ void ld128v(const uint64_t *p, uint64_t &x, uint64_t 
                      : "=l"(x), "=l"(y)
                      : "r"((unsigned)__cvta_generic_to_shared(p))
                      : "memory");
-}
-
-// Stored form of an inline key: word 1 is complemented, so a real key never reads (0, 0) = empty
-// (k <= 63 leaves at least two zero pad bits in word 1).
-template <int NW>
-__device__ __forceinline__ void inline_form(const KmerN<NW> &K, int KW, uint64_t &a, uint64_t &b) {
-    a = K.w[0];
-    b = ~(KW >= 2 ? K.w[1] : 0ull);
 }
 
 struct TabCtx {   // what a table operation needs
@@ -352,68 +384,20 @@ __device__ __forceinline__ void votes_of(const TabCtx &T, uint32_t s, uint32_t l
     }
 }
 
-// Inline-key tables probe linearly from an even slot, so that a probe round can test the slot pair
-// (s, s+1) with two adjacent 16 B loads (cap is even).
-__device__ __forceinline__ uint32_t slot0_inl(uint64_t h, uint32_t cap) { return slot_of(h, cap) & ~1u; }
-
-template <bool GT>
-__device__ __forceinline__ void slot_ld128(const TabCtx &T, size_t s, uint64_t &x, uint64_t &y) {
-    if (GT)
-        asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(x), "=l"(y) : "l"(T.keys + 2 * s) : "memory");
-    else
-        asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];"
-                     : "=l"(x), "=l"(y)
-                     : "r"(T.ks + 16u * (uint32_t)s)
-                     : "memory");
-}
-template <bool GT>
-__device__ __forceinline__ void slot_cas128(const TabCtx &T, size_t s, uint64_t n0, uint64_t n1, uint64_t &o0,
-                                            uint64_t &o1) {
-    if (GT) {
-        cas128<true>((void *)(T.keys + 2 * s), 0ull, 0ull, n0, n1, o0, o1);
-    } else {
-        asm volatile(
-            "{\n .reg .b128 d, b, c;\n mov.b128 b, {%2, %3};\n mov.b128 c, {%4, %5};\n"
-            " atom.shared.cas.b128 d, [%6], b, c;\n mov.b128 {%0, %1}, d;\n}"
-            : "=l"(o0), "=l"(o1)
-            : "l"(0ull), "l"(0ull), "l"(n0), "l"(n1), "r"(T.ks + 16u * (uint32_t)s)
-            : "memory");
-    }
-}
-template <bool GT>
-__device__ __forceinline__ uint64_t slot_ld_w0(const TabCtx &T, size_t s) {
-    uint64_t x;
-    if (GT)
-        asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(x) : "l"(T.keys + 2 * s) : "memory");
-    else
-        asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(x) : "r"(T.ks + 16u * (uint32_t)s) : "memory");
-    return x;
-}
-
+// Scalar lookup of a pointer-key (REF) table: the start k-mer
 template <bool INL, int NW>
 __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> &K, uint64_t h) {
-    uint32_t s = INL ? slot0_inl(h, T.cap) : slot_of(h, T.cap);
-    if (INL) {
-        uint64_t a, b;
-        inline_form(K, T.KW, a, b);
-        const ulonglong2 *kk = (const ulonglong2 *)T.keys;
-        for (uint32_t n = 0; n < T.cap; ++n) {
-            const ulonglong2 w = kk[s];
-            if (w.y == 0) return NONE;
-            if (w.x == a && w.y == b) return s;
-            s = (s + 1 == T.cap) ? 0 : s + 1;
+    static_assert(!INL, "inline-key tables use lookup32 (la_inl32.cuh)");
+    uint32_t s = slot_of(h, T.cap);
+    const uint64_t tag = tag_of(h);
+    for (uint32_t n = 0; n < T.cap; ++n) {
+        const uint64_t w = T.keys[s];
+        if (w == 0) return NONE;
+        if ((w & TAG_MASK) == tag) {
+            const KmerN<NW> K2 = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
+            if (kmer_eq(K, K2, T.KW)) return s;
         }
-    } else {
-        const uint64_t tag = tag_of(h);
-        for (uint32_t n = 0; n < T.cap; ++n) {
-            const uint64_t w = T.keys[s];
-            if (w == 0) return NONE;
-            if ((w & TAG_MASK) == tag) {
-                const KmerN<NW> K2 = extract_kmer<NW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), T.k, T.KW);
-                if (kmer_eq(K, K2, T.KW)) return s;
-            }
-            s = (s + 1 == T.cap) ? 0 : s + 1;
-        }
+        s = (s + 1 == T.cap) ? 0 : s + 1;
     }
     return NONE;
 }
@@ -427,181 +411,9 @@ __device__ unsigned long long g_probe_stats[8];
 #define LA_PSTAT(i, v) ((void)0)
 #endif
 
-// ---- warp-convergent passes (k <= 63, inline keys) --------------------------------------------
-// Lane-per-position: builder warp w owns the contiguous range [w*U/NW, (w+1)*U/NW) of the end's
-// numbered positions (pref, read by read) and its 32 lanes take 32 consecutive positions per
-// iteration, so every lane runs the same iteration count and the hash / probe / vote code executes
-// with the whole warp active (the per-thread rolling loops ran at ~5 of 32 lanes, ncu r01).  Each lane
-// extracts its k-mer from the packed read (3 words, funnel shifts) — no rolling, no read-boundary
-// branches; consecutive lanes read the same or adjacent words (broadcast).
-struct PosV {            // one lane's position
-    KmerN<2> K;
-    uint32_t nb;         // following base (Alg 1 line 6)
-    bool vote, hi;       // votes at all (q >= q_lo and no N in the window) / in the high tier
-};
-
+// ---- warp-convergent passes for pointer keys (k >= 64) ----------------------------------------
 __device__ __forceinline__ uint64_t nmask_word(uint64_t q) { return q & (q >> 1) & 0x5555555555555555ull; }
 
-// position p of read row (R, Q); has_n: the read contains an N (rflag); m0, m1: masks of the k-mer's
-// bits in its two words (hoisted out of the position loop)
-__device__ __forceinline__ PosV pos_value(const uint64_t *R, const uint64_t *Q, int p, int k, int SW, bool has_n,
-                                          uint64_t m0, uint64_t m1) {
-    PosV v;
-    const int q = p >> 5, s = (p & 31) << 1;
-    const int q2 = min(q + 2, SW - 1);   // word q+2 is only needed when the window reaches it
-    const uint64_t r0 = R[q], r1 = R[q + 1], r2 = R[q2];
-    v.K.w[0] = funnel64(r0, r1, s) & m0;
-    v.K.w[1] = funnel64(r1, r2, s) & m1;
-    const int i = p + k, wi = i >> 5, d = wi - q;   // following base, word q+d (d in 0..2)
-    const uint64_t rw = d == 0 ? r0 : (d == 1 ? r1 : r2);
-    const int sh = 62 - ((i & 31) << 1);
-    v.nb = (uint32_t)(rw >> sh) & 3u;
-    const uint32_t nq = (uint32_t)(Q[wi] >> sh) & 3u;
-    v.vote = nq - 1u < 2u;
-    v.hi = nq == 2u;
-    if (has_n) {   // reading #5: a k-mer with an N has no entry (rare: ~1% of reads)
-        const uint64_t n0 = nmask_word(Q[q]), n1 = nmask_word(Q[q + 1]), n2 = nmask_word(Q[q2]);
-        if ((funnel64(n0, n1, s) & m0) | (funnel64(n1, n2, s) & m1)) v.vote = false;
-    }
-    return v;
-}
-
-__device__ __forceinline__ void kmer_masks(int k, uint64_t &m0, uint64_t &m1) {
-    const int b1 = 2 * k - 64;   // bits of word 1 (<= 0: k <= 32)
-    m0 = b1 >= 0 ? ~0ull : (~0ull << (64 - 2 * k));
-    m1 = b1 > 0 ? (~0ull << (64 - b1)) : 0ull;
-}
-
-// f(act, v): act = this lane has a position this iteration (warp-uniform call).
-template <typename F>
-__device__ __forceinline__ void warp_positions(const uint64_t *__restrict__ rseq, const uint64_t *__restrict__ rqc,
-                                               const uint8_t *__restrict__ rflag, const uint32_t *pref,
-                                               long long r0, int r, int SW, int k, int KW, int wid, int nwarps,
-                                               int lane, const volatile int *stop, F &&f) {
-    (void)KW;
-    const uint32_t total = pref[r];
-    const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
-    const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
-    if (wb >= we) return;
-    uint64_t m0, m1;
-    kmer_masks(k, m0, m1);
-    uint32_t g = wb + lane;
-    int j;
-    {   // read j with pref[j] <= g < pref[j+1]
-        const uint32_t gg = min(g, we - 1);
-        int lo = 0, hi = r;
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (pref[mid] <= gg) lo = mid; else hi = mid;
-        }
-        j = lo;
-    }
-    // the lane's current read: position range [pj0, pj1), rows R / Q, has-N flag
-    uint32_t pj0 = pref[j], pj1 = pref[j + 1];
-    const uint64_t *R = rseq + (r0 + j) * SW, *Q = rqc + (r0 + j) * SW;
-    bool flag = rflag[r0 + j] != 0;
-    for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
-        if (((base - wb) & 127u) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;   // every 4th iteration
-        const bool act = g < we;
-        PosV v;
-        v.vote = false;
-        if (act) {
-            if (g >= pj1) {   // crossed into a later read (skips reads without positions)
-                do {
-                    pj0 = pj1;
-                    pj1 = pref[++j + 1];
-                } while (g >= pj1);
-                R = rseq + (r0 + j) * SW;
-                Q = rqc + (r0 + j) * SW;
-                flag = rflag[r0 + j] != 0;
-            }
-            v = pos_value(R, Q, (int)(g - pj0), k, SW, flag, m0, m1);
-        }
-        f(act && v.vote, v);
-    }
-}
-
-// Convergent insert of the lanes with `want` (Alg 1 line 5 + the vote): every probe round
-// is entered by the whole warp and tests a slot pair (s, s+1); claims are counted once per warp.
-// One slot of a round: 0 = resolved (found or claimed), 1 = occupied by another key, 2 = gave up
-// (overflow flagged), 3 = lost the claim race to another key (re-probe from this slot's successor).
-template <bool GT>
-__device__ __forceinline__ int probe_slot(const TabCtx &T, uint32_t s, uint64_t x, uint64_t y, uint64_t a, uint64_t bb,
-                                          bool &claimed, volatile int *ovf) {
-    if (y == 0) {   // looks empty: the CAS claims it or returns its true content
-        if (*ovf) return 2;
-        slot_cas128<GT>(T, s, a, bb, x, y);
-        if (y == 0) {
-            claimed = true;
-            return 0;
-        }
-        if (y == bb && x != a) x = slot_ld_w0<GT>(T, s);
-        return (x == a && y == bb) ? 0 : 3;
-    }
-    // a 16 B load is not single-copy atomic: if it raced with the claiming CAS, word 0 may be stale —
-    // re-read it (a slot never changes once claimed)
-    if (y == bb && x != a) x = slot_ld_w0<GT>(T, s);
-    return (x == a && y == bb) ? 0 : 1;
-}
-
-template <bool GT>
-__device__ __forceinline__ void warp_insert(const TabCtx &T, bool want, const PosV &v, uint64_t h, int lane,
-                                            int *nclaim, int claim_limit, volatile int *ovf) {
-    uint32_t s = slot0_inl(h, T.cap);
-    const uint64_t a = v.K.w[0], bb = ~(T.KW >= 2 ? v.K.w[1] : 0ull);
-    bool pend = want, found = false;
-    uint32_t hit = 0;
-#ifdef LA_PROBE_STATS
-    { const unsigned m = __ballot_sync(0xffffffffu, want); if (lane == 0) { LA_PSTAT(0, 1); LA_PSTAT(2, __popc(m)); } }
-#endif
-    while (__any_sync(0xffffffffu, pend)) {
-        if (lane == 0) LA_PSTAT(1, 1);
-        bool claimed = false;
-        if (pend) {
-            uint64_t x0, y0, x1, y1;
-            const uint32_t s1 = s + 1 == T.cap ? 0 : s + 1;   // s is even except after a lost claim race
-            slot_ld128<GT>(T, s, x0, y0);
-            slot_ld128<GT>(T, s1, x1, y1);
-            int st = probe_slot<GT>(T, s, x0, y0, a, bb, claimed, ovf);
-            if (st == 0) {
-                hit = s;
-                pend = false;
-                found = true;
-            } else if (st == 2) {
-                pend = false;
-            } else if (st == 3) {
-                s = s1;   // the slot pair loaded before the lost race may be stale: next round
-            } else {
-                st = probe_slot<GT>(T, s1, x1, y1, a, bb, claimed, ovf);
-                if (st == 0) {
-                    hit = s1;
-                    pend = false;
-                    found = true;
-                } else if (st == 2) {
-                    pend = false;
-                } else {
-                    s = s1 + 1 == T.cap ? 0 : s1 + 1;
-                }
-            }
-        }
-        const unsigned cm = __ballot_sync(0xffffffffu, claimed);
-        if (cm) {
-            const int n = __popc(cm), leader = __ffs(cm) - 1;
-            int first = 0;
-            if (lane == leader) {
-                LA_PSTAT(3, n);
-                first = atomicAdd(nclaim, n);
-                if (first + n > claim_limit) *ovf = 1;
-            }
-            first = __shfl_sync(0xffffffffu, first, leader);
-            // claims <= cap always (a claim takes an empty slot), so the list cannot overflow
-            if (claimed) T.list[first + __popc(cm & ((1u << lane) - 1u))] = (uint16_t)hit;
-        }
-    }
-    if (found) vote_add<GT>(T, hit, v.nb, v.hi, ovf);
-}
-
-// ---- warp-convergent passes for pointer keys (k >= 64) ----------------------------------------
 struct PosR {            // one lane's position, k-mer of up to 4 words
     KmerN<MAX_KW> K;
     uint32_t nb, rid;    // following base, read index (relative to the key rows)
@@ -753,42 +565,6 @@ __device__ __forceinline__ uint32_t warp_lookup_ref(const TabCtx &T, bool want, 
     return res;
 }
 
-// Convergent lookup (no insert): slot of K or NONE; slot pairs as in warp_insert.
-template <bool GT>
-__device__ __forceinline__ uint32_t warp_lookup(const TabCtx &T, bool want, const KmerN<2> &K, uint64_t h) {
-    uint32_t s = slot0_inl(h, T.cap), res = NONE;
-    const uint64_t a = K.w[0], bb = ~(T.KW >= 2 ? K.w[1] : 0ull);
-    bool pend = want;
-    uint32_t n = 0;
-#ifdef LA_PROBE_STATS
-    { const unsigned m = __ballot_sync(0xffffffffu, want); if ((threadIdx.x & 31) == 0) { LA_PSTAT(4, 1); LA_PSTAT(6, __popc(m)); } }
-#endif
-    while (__any_sync(0xffffffffu, pend)) {
-        if ((threadIdx.x & 31) == 0) LA_PSTAT(5, 1);
-        if (pend) {
-            uint64_t x0, y0, x1, y1;
-            slot_ld128<GT>(T, s, x0, y0);
-            slot_ld128<GT>(T, s + 1, x1, y1);   // s even, cap even: s+1 < cap
-            if (y0 == 0) {
-                pend = false;
-            } else if (x0 == a && y0 == bb) {
-                pend = false;
-                res = s;
-            } else if (y1 == 0) {
-                pend = false;
-            } else if (x1 == a && y1 == bb) {
-                pend = false;
-                res = s + 1;
-            } else {
-                s = s + 2 == T.cap ? 0 : s + 2;
-                n += 2;
-                if (n >= T.cap) pend = false;
-            }
-        }
-    }
-    return res;
-}
-
 // ---- the kernel --------------------------------------------------------------------------------
 struct EndSlot {            // one contig end in flight
     int e, r, ulen;         // ulen: common length of all the end's reads (0 if they differ)
@@ -797,6 +573,7 @@ struct EndSlot {            // one contig end in flight
     int best_len, best_term, best_k, best_buf;
     int done, dead, ovf;    // done: finished (refill); dead: no more ends; ovf: redo in the global path
     uint32_t start;         // the start k-mer's slot (NONE if absent) of the last build
+    int rec_att;            // replay: attempts recorded by the extension
     unsigned long long ins, steps;
 };
 
@@ -894,22 +671,195 @@ __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
     return (code < 4 ? (nxt == NONE ? NEXT_NONE : nxt) : NEXT_NONE) << 4 | (uint32_t)code;
 }
 
+// Inline keys (k <= 63) on 32-bit words (la_inl32.cuh): filter pass, build pass (Alg 1), link pass
+// (a5) and the start k-mer's slot, for NW = ceil(2k/32) words.
+template <int NW, bool GT>
+__device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, uint32_t *B1, uint32_t *B2,
+                                                 uint32_t mbits, uint32_t *info, const uint64_t *__restrict__ rqc,
+                                                 const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
+                                                 int r, int ulen, const DevParams &P, const uint64_t *tail_e, int Tn,
+                                                 uint64_t n0, uint64_t n1, int bt, int NB, long long &t_filter,
+                                                 long long &t_build, bool replay, void *fpos, uint32_t *queue) {
+    const volatile int *stop = &B.overflow;
+    const int k = TC.k;
+    const int lane = bt & 31, wid = bt >> 5, nwarps = NB >> 5;
+    const int claim_limit = (int)(SMEM_MAX_LOAD * (float)TC.cap);
+    Tab32 T;
+    T.keys = (unsigned char *)TC.keys;
+    T.ks = TC.ks;
+    T.c32 = TC.c32;
+    T.list = TC.list;
+    T.cap = TC.cap;
+    const uint32_t *R32 = (const uint32_t *)TC.rseq, *Q32 = (const uint32_t *)rqc;
+    const int SW2 = 2 * TC.SW;
+    if (!mbits || !LA_FQUEUE) {
+        if (mbits) {
+            // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
+            warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
+                                 [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
+                                     if (!act) return;
+                                     const uint32_t fi = filt32(h, mbits);
+                                     const uint32_t bit = 1u << (fi & 31);
+                                     if (!(*(volatile uint32_t *)&B2[fi >> 5] & bit)) {
+                                         if (LA_ABL_NOFILTATOM) {
+                                             const uint32_t old = B1[fi >> 5];
+                                             B1[fi >> 5] = old | bit;
+                                             if (old & bit) B2[fi >> 5] |= bit;
+                                         } else {
+                                             const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                             if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                                         }
+                                     }
+                                 });
+            builders_sync(NB);
+        }
+        t_filter = la_clock();
+        // ---- build (Alg 1): every voting occurrence that passed the filter ----
+        warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
+                             [&](bool, bool act, uint32_t, const K32<NW> &K, uint32_t h, uint32_t nb, bool hi) {
+                                 bool want = act;
+                                 if (mbits) {
+                                     const uint32_t fi = filt32(h, mbits);
+                                     want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+                                 }
+                                 warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim,
+                                                   claim_limit, &B.overflow);
+                             });
+    } else {
+        // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4); every position's
+        // filter bit index (or FNONE: no vote) is kept for the build pass ----
+        typedef typename std::conditional<GT, uint32_t, uint16_t>::type FT;
+        FT *fp = (FT *)fpos;
+        const uint32_t FNONE = GT ? 0xFFFFFFFFu : 0xFFFFu;
+        warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
+                             [&](bool inr, bool act, uint32_t g, const K32<NW> &, uint32_t h, uint32_t, bool) {
+                                 const uint32_t fi = filt32(h, mbits);
+                                 if (inr) fp[g] = (FT)(act ? fi : FNONE);
+                                 if (!act) return;
+                                 const uint32_t bit = 1u << (fi & 31);
+                                 if (!(*(volatile uint32_t *)&B2[fi >> 5] & bit)) {
+                                     const uint32_t old = atomicOr(&B1[fi >> 5], bit);
+                                     if (old & bit) atomicOr(&B2[fi >> 5], bit);
+                                 }
+                             });
+        builders_sync(NB);
+        t_filter = la_clock();
+        // ---- build (Alg 1): the positions whose filter bit is in B2 are queued per warp (64 slots
+        // in shared memory) and inserted 32 at a time, so the probe rounds run with full warps ----
+        const KMask m = kmask32<NW>(k);
+        const uint32_t total = pref[r];
+        const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
+        const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
+        auto insert_batch = [&](bool has, uint32_t g) {
+            int j = 0, p = 0;
+            if (has) pos_of(g, pref, r, ulen, k, j, p);
+            const long long row = (r0 + j) * (long long)SW2;
+            const uint32_t *Rr = R32 + row, *Qr = Q32 + row;
+            const K32<NW> K = extract32<NW>(Rr, p, m);
+            const uint32_t nb = base32(Rr, p + k), nq = base32(Qr, p + k);
+            const uint32_t h = hash32<NW>(K);
+            warp_insert32<GT>(T, has, key_form<NW>(K, h), h, nb, nq == 2u, lane, &B.nclaim, claim_limit, &B.overflow);
+        };
+        uint32_t qn = 0;   // queued positions (warp-uniform)
+        const unsigned lt = (1u << lane) - 1u;
+        for (uint32_t base = wb; base < we; base += 32u) {
+            if (((base - wb) & 127u) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) break;
+            const uint32_t g = base + lane;
+            bool want = false;
+            if (g < we) {
+                const uint32_t fi = fp[g];
+                want = fi != FNONE && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+            }
+            const unsigned wm = __ballot_sync(0xffffffffu, want);
+            if (want) queue[qn + __popc(wm & lt)] = g;
+            qn += __popc(wm);
+            if (qn >= 32u) {
+                __syncwarp();
+                const uint32_t gq = queue[lane], gx = queue[32 + lane];
+                __syncwarp();
+                if (lane < qn - 32u) queue[lane] = gx;
+                qn -= 32u;
+                insert_batch(true, gq);
+            }
+        }
+        __syncwarp();
+        if (__shfl_sync(0xffffffffu, *stop, 0) == 0 && qn) insert_batch(lane < qn, lane < qn ? queue[lane] : 0u);
+    }
+    builders_sync(NB);
+    t_build = la_clock();
+    if (B.overflow || replay) return;   // replay: the hash-build phase only (no link pass, no walk)
+    // ---- ext rule + successor links (a5), over the claimed slots, all lanes busy ----
+    const uint32_t nocc = min((uint32_t)B.nclaim, T.cap);
+    for (uint32_t base = (uint32_t)wid * 32u; base < nocc; base += (uint32_t)NB) {
+        const uint32_t i = base + lane;
+        const bool has = i < nocc;
+        const uint32_t s = has ? (uint32_t)T.list[i] : 0u;
+        K32<NW> K;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) K.w[w] = 0u;
+        int code = CODE_DEADEND;
+        if (has) {
+            K = key_of<NW>(ld_slot<GT>(T, s));
+            uint32_t lo[4], hi[4];
+            votes32<GT>(T, s, lo, hi);
+            code = ext_rule(lo, hi, P.V, P.F);
+            if (code < 4) roll32<NW>(K, k, (uint32_t)code);
+        }
+        const uint32_t h = hash32<NW>(K);
+        const uint32_t t = warp_lookup32<GT>(T, has && code < 4, key_form<NW>(K, h), h);
+        if (has) info[s] = link_info(code, t);
+    }
+    if (bt == 0) {
+        // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
+        const int p = Tn - k;
+        bool hasN = false;
+        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
+        uint32_t st = NONE;
+        if (!hasN) {
+            uint32_t Tw[2 * TAIL_W];
+#pragma unroll
+            for (int i = 0; i < TAIL_W; ++i) {
+                const uint64_t x = tail_e[i];
+                Tw[2 * i] = (uint32_t)x;
+                Tw[2 * i + 1] = (uint32_t)(x >> 32);
+            }
+            const K32<NW> K = extract32<NW>(Tw, p, kmask32<NW>(k));
+            const uint32_t h = hash32<NW>(K);
+            st = lookup32<GT>(T, key_form<NW>(K, h), h);
+        }
+        B.start = st;
+    }
+}
+
 template <bool INL, bool GT>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
                                            const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
                                            const uint32_t *pref, long long r0, int r, const DevParams &P,
                                            const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, int bt, int NB,
-                                           long long &t_filter, long long &t_build) {
+                                           long long &t_filter, long long &t_build, bool replay, int ulen, void *fpos,
+                                           uint32_t *queue) {
+    if (INL) {
+        const int nw = kw32(T.k);
+        if (nw <= 2)
+            inl32_build_link<2, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+        else if (nw == 3)
+            inl32_build_link<3, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+        else
+            inl32_build_link<4, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+        return;
+    }
+    // ---- pointer keys (k >= 64): the same passes with 4-word k-mers ----
     const volatile int *stop = &B.overflow;
     const int k = T.k, KW = T.KW;
     const int lane = bt & 31, wid = bt >> 5, nwarps = NB >> 5;
     const int claim_limit = (int)(SMEM_MAX_LOAD * (float)T.cap);
-    if (INL) {
-        // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
-        if (mbits) {
-            warp_positions(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
-                           [&](bool act, const PosV &v) {
+    if (mbits) {
+        warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                           [&](bool act, const PosR &v) {
                                if (!act) return;
                                const uint32_t fi = filt_index(hash_kmer(v.K, KW), mbits);
                                const uint32_t bit = 1u << (fi & 31);
@@ -918,82 +868,24 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                    if (old & bit) atomicOr(&B2[fi >> 5], bit);
                                }
                            });
-            builders_sync(NB);
-        }
-        t_filter = la_clock();
-        // ---- build (Alg 1) ----
-        {
-            warp_positions(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
-                      [&](bool act, const PosV &v) {
-                          const uint64_t h = hash_kmer(v.K, KW);
-                          bool want = act;
-                          if (mbits) {
-                              const uint32_t fi = filt_index(h, mbits);
-                              want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
-                          }
-                          warp_insert<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
-                      });
-        }
-    } else {
-        // ---- pointer keys (k >= 64): the same passes with 4-word k-mers ----
-        if (mbits) {
-            warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
-                               [&](bool act, const PosR &v) {
-                                   if (!act) return;
-                                   const uint32_t fi = filt_index(hash_kmer(v.K, KW), mbits);
-                                   const uint32_t bit = 1u << (fi & 31);
-                                   if (!(*(volatile uint32_t *)&B2[fi >> 5] & bit)) {
-                                       const uint32_t old = atomicOr(&B1[fi >> 5], bit);
-                                       if (old & bit) atomicOr(&B2[fi >> 5], bit);
-                                   }
-                               });
-            builders_sync(NB);
-        }
-        t_filter = la_clock();
-        warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
-                           [&](bool act, const PosR &v) {
-                               const uint64_t h = hash_kmer(v.K, KW);
-                               bool want = act;
-                               if (mbits) {
-                                   const uint32_t fi = filt_index(h, mbits);
-                                   want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
-                               }
-                               warp_insert_ref<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
-                           });
+        builders_sync(NB);
     }
+    t_filter = la_clock();
+    warp_positions_ref(T.rseq, rqc, rflag, pref, r0, r, T.SW, k, KW, wid, nwarps, lane, stop,
+                       [&](bool act, const PosR &v) {
+                           const uint64_t h = hash_kmer(v.K, KW);
+                           bool want = act;
+                           if (mbits) {
+                               const uint32_t fi = filt_index(h, mbits);
+                               want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+                           }
+                           warp_insert_ref<GT>(T, want, v, h, lane, &B.nclaim, claim_limit, &B.overflow);
+                       });
     builders_sync(NB);
     t_build = la_clock();
-    if (B.overflow) return;
-#ifdef LA_PROBE_STATS
-    if (bt == 0) LA_PSTAT(7, (unsigned long long)B.nclaim * 1000ull / T.cap);
-#endif
+    if (B.overflow || replay) return;   // replay: the hash-build phase only (no link pass, no walk)
     // ---- ext rule + successor links (a5) into the end's info buffer ----
-    if (INL) {
-        // Only occupied slots (~30% of the table) are visited: warp_insert appends every claimed slot
-        // to the claim list, so the warps take 32 list entries at a time with all lanes busy.
-        auto link_batch = [&](bool has, uint32_t s) {
-            KmerN<2> K;
-            K.w[0] = K.w[1] = 0;
-            int code = CODE_DEADEND;
-            if (has) {
-                const ulonglong2 w = ((const ulonglong2 *)T.keys)[s];
-                K.w[0] = w.x;
-                K.w[1] = KW >= 2 ? ~w.y : 0ull;
-                uint32_t lo[4], hi[4];
-                votes_of<GT>(T, s, lo, hi);
-                code = ext_rule(lo, hi, P.V, P.F);
-                if (code < 4) roll_kmer(K, k, KW, (uint32_t)code);
-            }
-            const uint32_t t = warp_lookup<GT>(T, has && code < 4, K, hash_kmer(K, KW));
-            if (has) info[s] = link_info(code, t);
-        };
-        // the claimed slots, in claim order (warp_insert), all lanes busy
-        const uint32_t nocc = min((uint32_t)B.nclaim, T.cap);
-        for (uint32_t base = (uint32_t)wid * 32u; base < nocc; base += (uint32_t)NB) {
-            const uint32_t i = base + lane;
-            link_batch(i < nocc, i < nocc ? (uint32_t)T.list[i] : 0u);
-        }
-    } else {
+    {
         const uint32_t nocc = min((uint32_t)B.nclaim, T.cap);
         for (uint32_t base = (uint32_t)wid * 32u; base < nocc; base += (uint32_t)NB) {
             const uint32_t i = base + lane;
@@ -1025,13 +917,8 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
             uint64_t Tw[TAIL_W];
 #pragma unroll
             for (int i = 0; i < TAIL_W; ++i) Tw[i] = tail_e[i];
-            if (INL) {
-                const KmerN<2> K = extract_kmer<2>(Tw, p, k, KW);
-                st = tab_lookup<true, 2>(T, K, hash_kmer(K, KW));
-            } else {
-                const KmerN<MAX_KW> K = extract_kmer<MAX_KW>(Tw, p, k, KW);
-                st = tab_lookup<false, MAX_KW>(T, K, hash_kmer(K, KW));
-            }
+            const KmerN<MAX_KW> K = extract_kmer<MAX_KW>(Tw, p, k, KW);
+            st = tab_lookup<false, MAX_KW>(T, K, hash_kmer(K, KW));
         }
         B.start = st;
     }
@@ -1047,7 +934,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     const uint64_t *__restrict__ tailN, const int32_t *__restrict__ clen, int SW, DevParams P,
     uint32_t smem_bytes, uint8_t *__restrict__ walk_buf, int32_t *__restrict__ out_len,
     uint8_t *__restrict__ out_term, uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
-    int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
+    int8_t *__restrict__ out_dir, int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
     unsigned char *__restrict__ gscratch, uint32_t gstride, unsigned long long *__restrict__ prof) {
     static_assert(BLOCK >= 64, "one walker warp + at least one builder warp");
     constexpr int NB = BLOCK - 32;   // builder threads
@@ -1055,9 +942,9 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     __shared__ EndSlot S[2];
     __shared__ BuildCtl B;
     __shared__ __align__(8) uint64_t built[2], walked[2];   // mbarriers: slot s built / walked
-    __shared__ unsigned long long s_acc[4];   // work counters: inserts, walk steps, attempts, filtered
+    __shared__ unsigned long long s_acc[GSTATS_WORDS];   // work counters (GlobalStats order)
     const int tid = threadIdx.x;
-    const SmemFixed FX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u);
+    const SmemFixed FX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u, false, NB / 32);
     // table region: shared memory, or this CTA's slice of the global scratch (XL class)
     unsigned char *tbase = GT ? gscratch + (size_t)blockIdx.x * gstride : sm;
     const int Wp = (P.W + 15) & ~15;
@@ -1070,7 +957,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             S[i].dead = 0;
             S[i].ovf = 0;
         }
-        for (int i = 0; i < 4; ++i) s_acc[i] = 0;
+        for (int i = 0; i < GSTATS_WORDS; ++i) s_acc[i] = 0;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -1101,7 +988,11 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             }
             int done = 0, bl = 0, bb = 0;
             const long long tw1 = la_clock();
-            if (lane == 0) {
+            if (lane == 0 && P.replay) {   // replay: the recorded k sequence instead of the walk
+                E.attempts += 1;
+                done = E.attempts >= E.rec_att;
+                E.k += E.shift;
+            } else if (lane == 0) {
                 // ---- walk (Alg 2) over the successor links ----
                 uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
                 uint8_t *wb = wstr + (2 * s + (E.best_buf ^ 1)) * Wp;
@@ -1139,7 +1030,13 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             bl = __shfl_sync(0xffffffffu, bl, 0);
             bb = __shfl_sync(0xffffffffu, bb, 0);
             w_walk += la_clock() - tw1;
-            if (done) {
+            if (done && P.replay) {
+                if (lane == 0) {
+                    s_acc[0] += E.ins;
+                    s_acc[2] += E.attempts;
+                    E.done = 1;
+                }
+            } else if (done) {
                 // ---- the selected walk -> HBM ----
                 const int e = E.e;
                 const uint8_t *bw = wstr + (2 * s + bb) * Wp;
@@ -1150,6 +1047,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                     out_term[e] = (uint8_t)E.best_term;
                     out_k[e] = (uint8_t)E.best_k;
                     out_att[e] = (uint8_t)E.attempts;
+                    out_dir[e] = shift_dir(E.shift);
                     s_acc[0] += E.ins;   // per-CTA work counters in shared memory (no registers)
                     s_acc[1] += E.steps;
                     s_acc[2] += E.attempts;
@@ -1189,13 +1087,16 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             B.overflow = 0;
             B.nclaim = 0;
             if (E.done) {   // refill the slot with the next end, or retire it
-                const int idx = atomicAdd(work_ctr, 1);
+                int idx, e = 0;
+                do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
+                    idx = atomicAdd(work_ctr, 1);
+                    if (idx < n_list) e = list[idx];
+                } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
                 if (idx >= n_list) {
                     E.dead = 1;
                     B.skip = 1;
                     mbar_arrive(&built[s]);   // the walker sees `dead` and retires the slot too
                 } else {
-                    const int e = list[idx];
                     E.e = e;
                     E.r0 = eoff[e];
                     E.r = (int)(eoff[e + 1] - E.r0);
@@ -1212,6 +1113,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                     E.steps = 0;
                     E.done = 0;
                     E.ovf = 0;
+                    if (P.replay) {
+                        E.rec_att = out_att[e];
+                        E.shift = out_dir[e] * P.k_shift;
+                    }
                 }
             }
         }
@@ -1307,12 +1212,16 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 TB.cap = (need + 1u) & ~1u;
                 TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
                 TB.off_list = TB.off_cnts + TB.cap * cnt_bytes(true);
+                TB.off_f = (TB.off_list + TB.cap * 2u + 15u) & ~15u;
             }
         }
         bool ovf = no_room || TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
         if (!ovf) {
             const uint32_t mbits = TB.mwords * 32u;
-            if (mbits && bt == 0) s_acc[3] += 1;
+            if (bt == 0) {
+                s_acc[3] += mbits ? 1 : 0;
+                s_acc[INL ? 4 : 5] += 1;
+            }
             uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);   // filters: always shared memory
             uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
             TabCtx T;
@@ -1341,12 +1250,15 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             const uint64_t *tail_e = tail + (size_t)e * TAIL_W;
             const uint64_t n0 = tailN[2 * (size_t)e], n1 = tailN[2 * (size_t)e + 1];
             uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
+            const int ulen_now = E.ulen;   // set by read_prefix (published by the barrier above)
+            void *fpos = GT ? (void *)(tbase + TB.off_f) : (void *)(sm + TB.off_f);
+            uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (INL)
                 build_link<true, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                     t_filter, t_build);
+                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
             else
                 build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                      t_filter, t_build);
+                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
         }
         builders_sync(NB);   // info buffer complete; the table is free for the next build
@@ -1361,7 +1273,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             if (ovf) {
                 // table or counter overflow: the global path redoes this end from scratch; the
                 // slot is refilled on its next turn (the walker only passes it through)
-                ovf_list[atomicAdd(n_ovf, 1)] = E.e;
+                if (!P.replay) {
+                    ovf_list[atomicAdd(n_ovf, 1)] = E.e;
+                    out_dir[E.e] = OVF_DIR;
+                }
                 E.ovf = 1;
                 E.done = 1;
             } else {
@@ -1373,6 +1288,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     }
     if (bt == 0) {
         atomicAdd(&gstats->filtered, s_acc[3]);
+        atomicAdd(&gstats->inl, s_acc[4]);
+        atomicAdd(&gstats->ref, s_acc[5]);
         if (prof)
             for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
     }
@@ -1394,7 +1311,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
     const uint64_t *__restrict__ tailN, const int32_t *__restrict__ clen, int SW, DevParams P,
     uint32_t smem_bytes, uint8_t *__restrict__ walk_buf, int32_t *__restrict__ out_len,
     uint8_t *__restrict__ out_term, uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
-    int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
+    int8_t *__restrict__ out_dir, int32_t *__restrict__ ovf_list, int *__restrict__ n_ovf, GlobalStats *__restrict__ gstats,
     unsigned char *__restrict__ gscratch, uint32_t gstride, unsigned long long *__restrict__ prof) {
     (void)gscratch;
     (void)gstride;
@@ -1403,21 +1320,24 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
     __shared__ EndSlot E;
     __shared__ BuildCtl B;
     __shared__ int s_done;
-    __shared__ unsigned long long s_acc[4];   // work counters: inserts, walk steps, attempts, filtered
+    __shared__ unsigned long long s_acc[GSTATS_WORDS];   // work counters (GlobalStats order)
     const int bt = threadIdx.x;
-    const SmemFixed FX = smem_fixed(P.W, smem_bytes, 0u, true);
+    const SmemFixed FX = smem_fixed(P.W, smem_bytes, 0u, true, NB / 32);
     const int Wp = (P.W + 15) & ~15;
     uint8_t *wstr = sm + FX.off_walk;   // two walk strings: current / best
     uint32_t *info = (uint32_t *)sm;
-    if (bt < 4) s_acc[bt] = 0;   // published by the first __syncthreads below
+    if (bt < GSTATS_WORDS) s_acc[bt] = 0;   // published by the first __syncthreads below
     long long b_t[8] = {0, 0, 0, 0, 0, 0, 0, 0};   // leader cycles: fetch, prefix, clear, filter, build, link, -, walk
     for (;;) {
         const long long ta = la_clock();
         if (bt == 0) {
-            const int idx = atomicAdd(work_ctr, 1);
+            int idx, e = 0;
+            do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
+                idx = atomicAdd(work_ctr, 1);
+                if (idx < n_list) e = list[idx];
+            } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
             B.skip = idx >= n_list;
             if (!B.skip) {
-                const int e = list[idx];
                 E.e = e;
                 E.r0 = eoff[e];
                 E.r = (int)(eoff[e + 1] - E.r0);
@@ -1432,6 +1352,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 E.best_buf = 1;
                 E.ins = 0;
                 E.steps = 0;
+                if (P.replay) {
+                    E.rec_att = out_att[e];
+                    E.shift = out_dir[e] * P.k_shift;
+                }
             }
         }
         __syncthreads();
@@ -1477,7 +1401,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 break;
             }
             const uint32_t mbits = TB.mwords * 32u;
-            if (mbits && bt == 0) s_acc[3] += 1;
+            if (bt == 0) {
+                s_acc[3] += mbits ? 1 : 0;
+                s_acc[inline_keys(k) ? 4 : 5] += 1;
+            }
             uint32_t *B1 = (uint32_t *)(sm + TB.off_b1);
             uint32_t *B2 = (uint32_t *)(sm + TB.off_b2);
             TabCtx T;
@@ -1505,12 +1432,15 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             __syncthreads();
             const long long td = la_clock();
             long long t_filter = td, t_build = td;
+            const int ulen_now = E.ulen;   // set by read_prefix (published by the barrier above)
+            void *fpos = (void *)(sm + TB.off_f);
+            uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (inline_keys(k))
                 build_link<true, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                        NB, t_filter, t_build);
+                                        NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
             else
                 build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                         NB, t_filter, t_build);
+                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
             __syncthreads();
             const long long te = la_clock();
             b_t[1] += tc - tb;
@@ -1522,7 +1452,12 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 ovf = true;
                 break;
             }
-            if (bt == 0) {
+            if (bt == 0 && P.replay) {   // replay: the recorded k sequence instead of the walk
+                E.ins += U;
+                E.attempts += 1;
+                s_done = E.attempts >= E.rec_att;
+                E.k += E.shift;
+            } else if (bt == 0) {
                 // ---- walk (Alg 2) over the successor links ----
                 E.ins += U;
                 uint8_t *wb = wstr + (E.best_buf ^ 1) * Wp;
@@ -1559,7 +1494,15 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             if (s_done) break;
         }
         if (ovf) {   // table or counter overflow: the global path redoes this end from scratch
-            if (bt == 0) ovf_list[atomicAdd(n_ovf, 1)] = e;
+            if (bt == 0 && !P.replay) {
+                ovf_list[atomicAdd(n_ovf, 1)] = e;
+                out_dir[e] = OVF_DIR;
+            }
+        } else if (P.replay) {
+            if (bt == 0) {
+                s_acc[0] += E.ins;
+                s_acc[2] += E.attempts;
+            }
         } else {
             const int bl = E.best_len;
             const uint8_t *bw = wstr + E.best_buf * Wp;
@@ -1570,6 +1513,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 out_term[e] = (uint8_t)E.best_term;
                 out_k[e] = (uint8_t)E.best_k;
                 out_att[e] = (uint8_t)E.attempts;
+                out_dir[e] = shift_dir(E.shift);
                 s_acc[0] += E.ins;
                 s_acc[1] += E.steps;
                 s_acc[2] += E.attempts;
@@ -1578,10 +1522,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
         __syncthreads();   // E and the staged reads are reused by the next end
     }
     if (bt == 0) {
-        atomicAdd(&gstats->inserts, s_acc[0]);
-        atomicAdd(&gstats->steps, s_acc[1]);
-        atomicAdd(&gstats->attempts, s_acc[2]);
-        atomicAdd(&gstats->filtered, s_acc[3]);
+        unsigned long long *g = &gstats->inserts;
+        for (int i = 0; i < GSTATS_WORDS; ++i) atomicAdd(&g[i], s_acc[i]);
         if (prof) {
             for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
             atomicAdd(&prof[7], (unsigned long long)b_t[7]);

@@ -59,20 +59,18 @@ namespace {
 using ClassKernel = void (*)(const int32_t *, int, int *, const uint64_t *, const uint64_t *, const uint16_t *,
                              const uint8_t *, const int64_t *, const uint64_t *, const uint64_t *, const int32_t *,
                              int, DevParams, uint32_t, uint8_t *, int32_t *, uint8_t *, uint8_t *, uint8_t *,
-                             int32_t *, int *, GlobalStats *, unsigned char *, uint32_t, unsigned long long *);
+                             int8_t *, int32_t *, int *, GlobalStats *, unsigned char *, uint32_t,
+                             unsigned long long *);
 struct ClassEntry {
     int threads, ctas;
     bool small;
     ClassKernel fn;
 };
-const ClassEntry kClassKernels[] = {
-    {64, 12, true, k_small<64, 12>},     {64, 16, true, k_small<64, 16>},     {96, 8, true, k_small<96, 8>},
-    {128, 6, true, k_small<128, 6>},     {128, 8, true, k_small<128, 8>},     {192, 4, true, k_small<192, 4>},
-    {256, 3, true, k_small<256, 3>},     {256, 4, true, k_small<256, 4>},
-    {128, 6, false, k_smem<128, false, 6>}, {192, 4, false, k_smem<192, false, 4>},
-    {256, 3, false, k_smem<256, false, 3>}, {256, 2, false, k_smem<256, false, 2>},
-    {256, 4, false, k_smem<256, false, 4>}, {384, 2, false, k_smem<384, false, 2>},
-    {512, 2, false, k_smem<512, false, 2>}, {512, 1, false, k_smem<512, false, 1>},
+const ClassEntry kClassKernels[] = {   // the five classes la_create configures (see cls_threads / cls_ctas)
+    {64, 12, true, k_small<64, 12>},
+    {128, 6, true, k_small<128, 6>},
+    {256, 3, false, k_smem<256, false, 3>},
+    {512, 2, false, k_smem<512, false, 2>},
     {1024, 1, false, k_smem<1024, false, 1>},
 };
 const ClassEntry *find_class_kernel(int threads, int ctas, bool small) {
@@ -104,7 +102,11 @@ struct la_ctx {
         smem_key2, glob_list, ctrs, ext_off, ext_seq, gstats, cub_tmp;
     DevBuf g_state, g_act, g_act2, g_still, g_cap, g_nrd, g_capoff, g_rdoff, g_slots, g_cnt, g_vis,
         g_cur;
-    DevBuf lens64, xl_scratch, prof;
+    DevBuf lens64, xl_scratch, prof, out_dir, hist;
+    // plan of the last la_extend (la_replay_build reruns its class lists)
+    bool extended = false;
+    int plan_ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
+    int plan_nxl = 0, plan_xl_umax = 0, plan_xl_rmax = 0;
     HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
     // la_extend_streamed: copy stream, double-buffered raw staging (A/B), chunk-ordering events
     cudaStream_t copy_stream = nullptr;
@@ -112,6 +114,7 @@ struct la_ctx {
     cudaEvent_t ev_copied[2] = {}, ev_loaded[2] = {};
     int64_t g_attempts = 0;
     cudaEvent_t ev[6] = {};
+    cudaEvent_t ev_rep[2] = {};   // la_replay_build start / end
     cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] classes may start
     cudaEvent_t ev_cls0[N_SMEM_CLASSES + 1] = {};  // start of class c ([N] = XL)
     // one stream per table class: the persistent class kernels are launched together (largest tables
@@ -272,10 +275,7 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         ctx->own_stream = true;
     }
     for (auto &e : ctx->ev) cudaEventCreate(&e);
-    for (auto &e : ctx->ev_cls0)
-        if (e) cudaEventDestroy(e);
-    for (auto &q : ctx->cls_stream)
-        if (q) cudaStreamDestroy(q);
+    for (auto &e : ctx->ev_rep) cudaEventCreate(&e);
     for (auto &e : ctx->ev_cls) cudaEventCreate(&e);
     for (auto &e : ctx->ev_cls0) cudaEventCreate(&e);
     for (auto &q : ctx->cls_stream)
@@ -323,13 +323,22 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
                       &ctx->glob_list, &ctx->ctrs, &ctx->ext_off, &ctx->ext_seq, &ctx->gstats,
                       &ctx->cub_tmp, &ctx->g_state, &ctx->g_act, &ctx->g_act2, &ctx->g_still, &ctx->g_cap,
                       &ctx->g_nrd, &ctx->g_capoff, &ctx->g_rdoff, &ctx->g_slots, &ctx->g_cnt, &ctx->g_vis,
-                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch, &ctx->prof})
+                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch, &ctx->prof, &ctx->out_dir, &ctx->hist})
         b->release();
     for (HostBuf *b : {&ctx->h_ext_off, &ctx->h_ext_seq, &ctx->h_term, &ctx->h_k, &ctx->h_att, &ctx->h_small})
         b->release();
     for (auto &e : ctx->ev)
         if (e) cudaEventDestroy(e);
+    for (auto &e : ctx->ev_rep)
+        if (e) cudaEventDestroy(e);
+    for (auto &q : ctx->cls_stream)
+        if (q) {
+            cudaStreamSynchronize(q);
+            cudaStreamDestroy(q);
+        }
     for (auto &e : ctx->ev_cls)
+        if (e) cudaEventDestroy(e);
+    for (auto &e : ctx->ev_cls0)
         if (e) cudaEventDestroy(e);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
     delete ctx;
@@ -465,7 +474,7 @@ extern "C" la_status la_load_batch(la_ctx *ctx, const la_batch *b, const la_para
         CK(grow(E.tailN, std::max<int64_t>(nE, 1) * 16));
         CK(grow(E.clen, std::max<int64_t>(nE, 1) * 4));
         DevParams dp{params->k_start, params->k_min, params->k_max, params->k_shift, params->max_walk_len,
-                     params->qual_offset, params->q_lo, params->q_hi, params->min_votes, params->min_frac_pct};
+                     params->qual_offset, params->q_lo, params->q_hi, params->min_votes, params->min_frac_pct, 0};
         if (nR) {
             CK(cudaMemsetAsync(E.rflag.p, 0, nR, st));
             k_read_end<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(E.eoff), nE, nR, P<int32_t>(ctx->read_end));
@@ -493,6 +502,7 @@ extern "C" la_status la_load_batch(la_ctx *ctx, const la_batch *b, const la_para
     std::swap(ctx->enc, ctx->spare);
     ctx->params = *params;
     ctx->loaded = true;
+    ctx->extended = false;
     return LA_OK;
 }
 
@@ -597,6 +607,82 @@ la_status run_global(la_ctx *ctx, const int32_t *d_list, int n_list, double *ms_
     return LA_OK;
 }
 
+// The table-class kernels over the plan's class lists (XL + the five shared-memory classes), on
+// one stream per class (LA_SERIAL_CLASSES=1: all on the context stream), joined back into the
+// context stream.  replay = true: la_replay_build's build-only pass over the same lists.
+la_status launch_classes(la_ctx *ctx, bool replay) {
+    cudaStream_t st = ctx->stream;
+    Encoded &E = ctx->enc;
+    DevParams dp = ctx->dp;
+    dp.replay = replay ? 1 : 0;
+    const int64_t nE = E.n_ends;
+    int *d_ctr = P<int>(ctx->ctrs);
+    unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
+    int32_t *lists = P<int32_t>(ctx->smem_list);
+    int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
+    const int n_xl = ctx->plan_nxl;
+    // LA_PROFILE=1: per-class phase cycle counters (clock64) of the shared-memory kernels
+    unsigned long long *prof = nullptr;
+    if (!replay && getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE"))) {
+        CK(grow(ctx->prof, 8 * 8 * (N_SMEM_CLASSES + 1)));
+        prof = P<unsigned long long>(ctx->prof);
+        CK(cudaMemsetAsync(prof, 0, 8 * 8 * (N_SMEM_CLASSES + 1), st));
+    }
+    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES + 1], st));
+    auto cls_st = [&](int c) -> cudaStream_t {
+        return (ctx->concurrent_classes && ctx->cls_stream[c]) ? ctx->cls_stream[c] : st;
+    };
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c)
+        if (cls_st(c) != st) CK(cudaStreamWaitEvent(cls_st(c), ctx->ev_cls[N_SMEM_CLASSES + 1], 0));
+    // XL (global-scratch tables) first, then the shared-memory classes from the largest tables
+    // (1 CTA/SM, all shared memory) to the smallest (12 CTAs/SM)
+    CK(cudaEventRecord(ctx->ev_cls0[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));
+    if (n_xl > 0) {
+        cudaStream_t sx = cls_st(N_SMEM_CLASSES);
+        const uint32_t bytes = ctx->xl_bytes;
+        const uint32_t icap = smem_fixed(dp.W, bytes, 1u, false, XL_THREADS / 32 - 1).icap;
+        const uint32_t stride = xl_stride(ctx->plan_xl_rmax, ctx->plan_xl_umax, dp.V >= 2, icap);
+        const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm, n_xl);
+        CK(grow(ctx->xl_scratch, (size_t)grid * stride));
+        int32_t *lst = lists + (size_t)N_SMEM_CLASSES * nE;
+        k_smem<XL_THREADS, true><<<grid, XL_THREADS, bytes, sx>>>(
+            lst, n_xl, d_ctr + 21, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
+            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
+            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
+            P<uint8_t>(ctx->out_att), P<int8_t>(ctx->out_dir), ovf_list, d_ctr + 15,
+            (GlobalStats *)(d_gst + 8 + GSTATS_WORDS * N_SMEM_CLASSES), P<unsigned char>(ctx->xl_scratch), stride,
+            prof ? prof + 8 * N_SMEM_CLASSES : nullptr);
+        CKL();
+        ctx->stats.ends_xl = n_xl;
+        ctx->stats.xl_scratch_bytes = (int64_t)grid * stride;
+    }
+    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));   // end of XL
+    for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
+        const int n = ctx->plan_ncls[c];
+        CK(cudaEventRecord(ctx->ev_cls0[c], cls_st(c)));
+        if (n > 0) {
+            cudaStream_t sc = cls_st(c);
+            const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm * ctx->cls_ctas[c], n);
+            const uint32_t bytes = ctx->cls_bytes[c];
+            int32_t *lst = lists + (size_t)c * nE;
+            int *wc = d_ctr + 16 + c;
+            const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], (ctx->small_mask >> c) & 1u);
+            if (!ke) return fail(ctx, LA_ERR_STATE, "no kernel instantiation for table class %d", c);
+            ke->fn<<<grid, ke->threads, bytes, sc>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
+                P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
+                P<int32_t>(E.clen), E.SW, dp, bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+                P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), P<int8_t>(ctx->out_dir),
+                ovf_list, d_ctr + 15, (GlobalStats *)(d_gst + 8 + GSTATS_WORDS * c), nullptr, 0u,
+                prof ? prof + 8 * c : nullptr);
+            CKL();
+        }
+        CK(cudaEventRecord(ctx->ev_cls[c], cls_st(c)));   // end of class c
+    }
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c)   // join
+        if (cls_st(c) != st) CK(cudaStreamWaitEvent(st, ctx->ev_cls[c], 0));
+    return LA_OK;
+}
+
 la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     if (!ctx || !out) return LA_ERR_INVALID_ARG;
     if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
@@ -625,6 +711,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
     CK(grow(ctx->ctrs, 256));
     CK(grow(ctx->gstats, 512));
+    CK(grow(ctx->out_dir, std::max<int64_t>(nE, 1)));
+    CK(grow(ctx->hist, 8 * LA_HIST));
     CK(grow(ctx->ext_off, (nE + 1) * 8));
     CK(grow_host(ctx->h_small, 1024));
     int *d_ctr = P<int>(ctx->ctrs);   // [0..4] n per class [5] n_G [6] NOREADS [7] SHORT [15] n_ovf [16..20] work
@@ -650,9 +738,11 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         }
         pb.single = ctx->small_mask;
         if (force_smem) pb.b[0] = 0xffffffffu;
+        // test hook: every end with reads into table class LA_FORCE_CLASS (0..4 shared memory, 5 = XL)
+        const int force_cls = getenv("LA_FORCE_CLASS") ? std::min(std::max(atoi(getenv("LA_FORCE_CLASS")), 0), 5) : -1;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
             P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
-            (force_global || force_smem) ? 0u : ctx->xl_bytes, P<int32_t>(ctx->cls),
+            (force_global || force_smem) ? 0u : ctx->xl_bytes, force_global ? -1 : force_cls, P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
             lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
@@ -682,64 +772,15 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         CK(cudaMemcpyAsync(lst, ctx->smem_list2.p, (size_t)n * 4, cudaMemcpyDeviceToDevice, st));
     }
     CK(cudaEventRecord(ctx->ev[1], st));
+    ctx->plan_nxl = n_xl;
+    ctx->plan_xl_umax = xl_umax;
+    ctx->plan_xl_rmax = xl_rmax;
+    for (int c = 0; c < N_SMEM_CLASSES; ++c) ctx->plan_ncls[c] = ncls[c];
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
-    // XL (global-scratch tables) first, then the shared-memory classes from the largest tables
-    // (1 CTA/SM, all shared memory) to the smallest (12 CTAs/SM)
-    // LA_PROFILE=1: per-class phase cycle counters (clock64) of the shared-memory kernels
-    unsigned long long *prof = nullptr;
-    if (getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE"))) {
-        CK(grow(ctx->prof, 8 * 8 * (N_SMEM_CLASSES + 1)));
-        prof = P<unsigned long long>(ctx->prof);
-        CK(cudaMemsetAsync(prof, 0, 8 * 8 * (N_SMEM_CLASSES + 1), st));
+    {
+        const la_status s0 = launch_classes(ctx, false);
+        if (s0 != LA_OK) return s0;
     }
-    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES + 1], st));
-    auto cls_st = [&](int c) -> cudaStream_t {
-        return (ctx->concurrent_classes && ctx->cls_stream[c]) ? ctx->cls_stream[c] : st;
-    };
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c)
-        if (cls_st(c) != st) CK(cudaStreamWaitEvent(cls_st(c), ctx->ev_cls[N_SMEM_CLASSES + 1], 0));
-    CK(cudaEventRecord(ctx->ev_cls0[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));
-    if (n_xl > 0) {
-        cudaStream_t st = cls_st(N_SMEM_CLASSES);
-        const uint32_t bytes = ctx->xl_bytes;
-        const uint32_t icap = smem_fixed(dp.W, bytes, 1u).icap;
-        const uint32_t stride = xl_stride(xl_rmax, xl_umax, dp.V >= 2, icap);
-        const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm, n_xl);
-        CK(grow(ctx->xl_scratch, (size_t)grid * stride));
-        int32_t *lst = lists + (size_t)N_SMEM_CLASSES * nE;
-        k_smem<XL_THREADS, true><<<grid, XL_THREADS, bytes, st>>>(
-            lst, n_xl, d_ctr + 21, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc), P<uint16_t>(E.rlen), P<uint8_t>(E.rflag),
-            P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), E.SW, dp, bytes,
-            P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k),
-            P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15, (GlobalStats *)(d_gst + 8 + 4 * N_SMEM_CLASSES),
-            P<unsigned char>(ctx->xl_scratch), stride, prof ? prof + 8 * N_SMEM_CLASSES : nullptr);
-        CKL();
-        ctx->stats.ends_xl = n_xl;
-        ctx->stats.xl_scratch_bytes = (int64_t)grid * stride;
-    }
-    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));   // end of XL
-    for (int c = N_SMEM_CLASSES - 1; c >= 0; --c) {
-        const int n = ncls[c];
-        CK(cudaEventRecord(ctx->ev_cls0[c], cls_st(c)));
-        if (n > 0) {
-            cudaStream_t st = cls_st(c);
-            const int grid = (int)std::min<int64_t>((int64_t)ctx->n_sm * ctx->cls_ctas[c], n);
-            const uint32_t bytes = ctx->cls_bytes[c];
-            int32_t *lst = lists + (size_t)c * nE;
-            int *wc = d_ctr + 16 + c;
-const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], (ctx->small_mask >> c) & 1u);
-            if (!ke) return fail(ctx, LA_ERR_STATE, "no kernel instantiation for table class %d", c);
-            ke->fn<<<grid, ke->threads, bytes, st>>>(lst, n, wc, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
-                P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
-                P<int32_t>(E.clen), E.SW, dp, bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
-                P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), ovf_list, d_ctr + 15,
-                (GlobalStats *)(d_gst + 8 + 4 * c), nullptr, 0u, prof ? prof + 8 * c : nullptr);
-            CKL();
-        }
-        CK(cudaEventRecord(ctx->ev_cls[c], cls_st(c)));   // end of class c
-    }
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c)   // join
-        if (cls_st(c) != st) CK(cudaStreamWaitEvent(st, ctx->ev_cls[c], 0));
     int n_ovf = 0;
     int n_smem = n_xl;
     for (int c = 0; c < N_SMEM_CLASSES; ++c) n_smem += ncls[c];
@@ -760,6 +801,11 @@ const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], 
         CK(grow(ctx->lens64, (nE + 1) * 8));
         k_len64<<<blocks(nE + 1, 256), 256, 0, st>>>(P<int32_t>(ctx->out_len), nE, P<int64_t>(ctx->lens64));
         CKL();
+        CK(cudaMemsetAsync(ctx->hist.p, 0, 8 * LA_HIST, st));
+        if (nE) {
+            k_att_hist<<<blocks(nE, 256), 256, 0, st>>>(P<uint8_t>(ctx->out_att), nE, P<unsigned long long>(ctx->hist));
+            CKL();
+        }
         size_t tb = 0;
         cub::DeviceScan::ExclusiveSum(nullptr, tb, P<int64_t>(ctx->lens64), P<int64_t>(ctx->ext_off), nE + 1, st);
         CK(grow(ctx->cub_tmp, tb));
@@ -768,18 +814,22 @@ const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], 
     }
     int64_t *h64 = (int64_t *)ctx->h_small.p;
     CK(cudaMemcpyAsync(h64, P<int64_t>(ctx->ext_off) + nE, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(h64 + 1, d_gst, 8 * (8 + 4 * (N_SMEM_CLASSES + 1)), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64 + 1, d_gst, 8 * (8 + GSTATS_WORDS * (N_SMEM_CLASSES + 1)), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64 + 64, ctx->hist.p, 8 * LA_HIST, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
-    if (prof) {
-        CK(cudaMemcpy(ctx->stats.prof_cycles, prof, sizeof(ctx->stats.prof_cycles), cudaMemcpyDeviceToHost));
+    if (getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE")) && ctx->prof.p) {
+        CK(cudaMemcpy(ctx->stats.prof_cycles, ctx->prof.p, sizeof(ctx->stats.prof_cycles), cudaMemcpyDeviceToHost));
     }
     // per-class stats (classes 0..4 shared memory, 5 = XL); fold them into the smem totals
+    for (int i = 0; i < LA_HIST; ++i) ctx->stats.attempts_hist[i] = h64[64 + i];
     for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
-        const int64_t *g = h64 + 1 + 8 + 4 * c;
+        const int64_t *g = h64 + 1 + 8 + GSTATS_WORDS * c;
         ctx->stats.cls_ends[c] = c < N_SMEM_CLASSES ? ncls[c] : n_xl;
         ctx->stats.cls_inserts[c] = g[0];
         ctx->stats.cls_attempts[c] = g[2];
         ctx->stats.cls_filtered[c] = g[3];
+        ctx->stats.cls_inl_attempts[c] = g[4];
+        ctx->stats.cls_ref_attempts[c] = g[5];
         h64[1] += g[0];
         h64[2] += g[1];
         h64[3] += g[2];
@@ -845,6 +895,9 @@ const ClassEntry *ke = find_class_kernel(ctx->cls_threads[c], ctx->cls_ctas[c], 
     ctx->stats.ends_by_class[4] = n_ovf;
     ctx->stats.ends_medium = ncls[3] + ncls[4];
     ctx->stats.ms_smem_medium = ctx->stats.cls_ms[N_SMEM_CLASSES] + ctx->stats.cls_ms[3] + ctx->stats.cls_ms[4];
+    ctx->stats.ms_build = -1.0;   // set by la_replay_build
+    ctx->stats.ms_walk = -1.0;
+    ctx->extended = true;
     return LA_OK;
 }
 
@@ -959,79 +1012,93 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
         CK(cudaEventRecord(ctx->ev_copied[i], cs));
         return LA_OK;
     };
-    la_status s;
-    if ((s = enqueue_copy(0))) return s;
-    if (nchunk > 1 && (s = enqueue_copy(1))) return s;
     la_stats acc{};
-    int64_t bases = 0;
-    for (int c = 0; c < nchunk; ++c) {
-        const int i = c & 1;
-        const Chunk k = chunk(c);
-        const int64_t nc = k.c1 - k.c0, nr = k.r1 - k.r0;
-        CK(cudaStreamWaitEvent(st, ctx->ev_copied[i], 0));
-        k_rebase<<<blocks(nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_coff[i]), nc + 1, k.s0);
-        k_rebase<<<blocks(nr + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_roff[i]), nr + 1, k.b0);
-        k_rebase<<<blocks(2 * nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_eoff[i]), 2 * nc + 1, k.r0);
-        CK(cudaGetLastError());
-        la_batch sub{};
-        sub.mem = LA_MEM_DEVICE;
-        sub.n_contigs = (int32_t)nc;
-        sub.contig_seq = P<char>(ctx->st_cseq[i]);
-        sub.contig_off = P<int64_t>(ctx->st_coff[i]);
-        sub.n_reads = nr;
-        sub.read_seq = P<char>(ctx->st_seq[i]);
-        sub.read_qual = P<char>(ctx->st_qual[i]);
-        sub.read_off = P<int64_t>(ctx->st_roff[i]);
-        sub.end_read_off = P<int64_t>(ctx->st_eoff[i]);
-        if ((s = la_load_batch(ctx, &sub, params))) return s;
-        CK(cudaEventRecord(ctx->ev_loaded[i], st));   // staging buffer i may be refilled
-        if (c + 2 < nchunk && (s = enqueue_copy(c + 2))) return s;
-        la_result r{};
-        if ((s = extend_impl(ctx, &r, false))) return s;
-        const int64_t ne = 2 * nc, nb = ctx->stats.ext_bases;
-        // results of this chunk -> the combined host buffers (device-side rebase of ext_off)
-        CK(grow(ctx->lens64, (ne + 1) * 8));
-        k_add_i64<<<blocks(ne + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->ext_off), ne + 1, bases, P<int64_t>(ctx->lens64));
-        CK(cudaGetLastError());
-        const int64_t e0 = 2 * k.c0;
-        CK(cudaMemcpyAsync(h_off + e0 + 1, P<int64_t>(ctx->lens64) + 1, ne * 8, cudaMemcpyDeviceToHost, st));
-        if (nb) CK(cudaMemcpyAsync((char *)ctx->h_ext_seq.p + bases, ctx->ext_seq.p, nb, cudaMemcpyDeviceToHost, st));
-        if (ne) {
-            CK(cudaMemcpyAsync((uint8_t *)ctx->h_term.p + e0, ctx->out_term.p, ne, cudaMemcpyDeviceToHost, st));
-            CK(cudaMemcpyAsync((uint8_t *)ctx->h_k.p + e0, ctx->out_k.p, ne, cudaMemcpyDeviceToHost, st));
-            CK(cudaMemcpyAsync((uint8_t *)ctx->h_att.p + e0, ctx->out_att.p, ne, cudaMemcpyDeviceToHost, st));
+    // every error return after the first enqueue_copy first drains the copy stream, so the caller's
+    // (pinned) host buffers are no longer read by queued DMA when la_extend_streamed returns
+    const la_status run = [&]() -> la_status {
+        la_status s;
+        if ((s = enqueue_copy(0))) return s;
+        if (nchunk > 1 && (s = enqueue_copy(1))) return s;
+        int64_t bases = 0;
+        for (int c = 0; c < nchunk; ++c) {
+            const int i = c & 1;
+            const Chunk k = chunk(c);
+            const int64_t nc = k.c1 - k.c0, nr = k.r1 - k.r0;
+            CK(cudaStreamWaitEvent(st, ctx->ev_copied[i], 0));
+            k_rebase<<<blocks(nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_coff[i]), nc + 1, k.s0);
+            k_rebase<<<blocks(nr + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_roff[i]), nr + 1, k.b0);
+            k_rebase<<<blocks(2 * nc + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->st_eoff[i]), 2 * nc + 1, k.r0);
+            CK(cudaGetLastError());
+            la_batch sub{};
+            sub.mem = LA_MEM_DEVICE;
+            sub.n_contigs = (int32_t)nc;
+            sub.contig_seq = P<char>(ctx->st_cseq[i]);
+            sub.contig_off = P<int64_t>(ctx->st_coff[i]);
+            sub.n_reads = nr;
+            sub.read_seq = P<char>(ctx->st_seq[i]);
+            sub.read_qual = P<char>(ctx->st_qual[i]);
+            sub.read_off = P<int64_t>(ctx->st_roff[i]);
+            sub.end_read_off = P<int64_t>(ctx->st_eoff[i]);
+            if ((s = la_load_batch(ctx, &sub, params))) return s;
+            CK(cudaEventRecord(ctx->ev_loaded[i], st));   // staging buffer i may be refilled
+            if (c + 2 < nchunk && (s = enqueue_copy(c + 2))) return s;
+            la_result r{};
+            if ((s = extend_impl(ctx, &r, false))) return s;
+            const int64_t ne = 2 * nc, nb = ctx->stats.ext_bases;
+            // results of this chunk -> the combined host buffers (device-side rebase of ext_off)
+            CK(grow(ctx->lens64, (ne + 1) * 8));
+            k_add_i64<<<blocks(ne + 1, 256), 256, 0, st>>>(P<int64_t>(ctx->ext_off), ne + 1, bases, P<int64_t>(ctx->lens64));
+            CK(cudaGetLastError());
+            const int64_t e0 = 2 * k.c0;
+            CK(cudaMemcpyAsync(h_off + e0 + 1, P<int64_t>(ctx->lens64) + 1, ne * 8, cudaMemcpyDeviceToHost, st));
+            if (nb) CK(cudaMemcpyAsync((char *)ctx->h_ext_seq.p + bases, ctx->ext_seq.p, nb, cudaMemcpyDeviceToHost, st));
+            if (ne) {
+                CK(cudaMemcpyAsync((uint8_t *)ctx->h_term.p + e0, ctx->out_term.p, ne, cudaMemcpyDeviceToHost, st));
+                CK(cudaMemcpyAsync((uint8_t *)ctx->h_k.p + e0, ctx->out_k.p, ne, cudaMemcpyDeviceToHost, st));
+                CK(cudaMemcpyAsync((uint8_t *)ctx->h_att.p + e0, ctx->out_att.p, ne, cudaMemcpyDeviceToHost, st));
+            }
+            bases += nb;
+            // accumulate the work and device-time counters over chunks
+            const la_stats &x = ctx->stats;
+            acc.ms_total += x.ms_total;
+            acc.ms_smem += x.ms_smem;
+            acc.ms_global += x.ms_global;
+            acc.ms_emit += x.ms_emit;
+            acc.inserts += x.inserts;
+            acc.inserts_smem += x.inserts_smem;
+            acc.walk_steps += x.walk_steps;
+            acc.attempts += x.attempts;
+            acc.ext_bases += x.ext_bases;
+            for (int q = 0; q < 5; ++q) acc.ends_by_class[q] += x.ends_by_class[q];
+            acc.kernel_launches += x.kernel_launches + 4;   // + the rebase / offset kernels
+            acc.global_rounds += x.global_rounds;
+            acc.ends_medium += x.ends_medium;
+            acc.ms_smem_medium += x.ms_smem_medium;
+            acc.ends_xl += x.ends_xl;
+            acc.xl_scratch_bytes = std::max(acc.xl_scratch_bytes, x.xl_scratch_bytes);
+            for (int q = 0; q < 6; ++q) {
+                acc.cls_ends[q] += x.cls_ends[q];
+                acc.cls_inserts[q] += x.cls_inserts[q];
+                acc.cls_attempts[q] += x.cls_attempts[q];
+                acc.cls_filtered[q] += x.cls_filtered[q];
+                acc.cls_inl_attempts[q] += x.cls_inl_attempts[q];
+                acc.cls_ref_attempts[q] += x.cls_ref_attempts[q];
+                acc.cls_ms[q] += x.cls_ms[q];
+            }
+            for (int q = 0; q < LA_HIST; ++q) acc.attempts_hist[q] += x.attempts_hist[q];
+            acc.smem_bytes_per_cta = x.smem_bytes_per_cta;
+            acc.smem_ctas_per_sm = x.smem_ctas_per_sm;
         }
-        bases += nb;
-        // accumulate the work and device-time counters over chunks
-        const la_stats &x = ctx->stats;
-        acc.ms_total += x.ms_total;
-        acc.ms_smem += x.ms_smem;
-        acc.ms_global += x.ms_global;
-        acc.ms_emit += x.ms_emit;
-        acc.inserts += x.inserts;
-        acc.inserts_smem += x.inserts_smem;
-        acc.walk_steps += x.walk_steps;
-        acc.attempts += x.attempts;
-        acc.ext_bases += x.ext_bases;
-        for (int q = 0; q < 5; ++q) acc.ends_by_class[q] += x.ends_by_class[q];
-        acc.kernel_launches += x.kernel_launches + 4;   // + the rebase / offset kernels
-        acc.global_rounds += x.global_rounds;
-        acc.ends_medium += x.ends_medium;
-        acc.ms_smem_medium += x.ms_smem_medium;
-        acc.ends_xl += x.ends_xl;
-        acc.xl_scratch_bytes = std::max(acc.xl_scratch_bytes, x.xl_scratch_bytes);
-        for (int q = 0; q < 6; ++q) {
-            acc.cls_ends[q] += x.cls_ends[q];
-            acc.cls_inserts[q] += x.cls_inserts[q];
-            acc.cls_attempts[q] += x.cls_attempts[q];
-            acc.cls_filtered[q] += x.cls_filtered[q];
-            acc.cls_ms[q] += x.cls_ms[q];
-        }
-        acc.smem_bytes_per_cta = x.smem_bytes_per_cta;
-        acc.smem_ctas_per_sm = x.smem_ctas_per_sm;
+        CK(cudaStreamSynchronize(st));
+        return LA_OK;
+    }();
+    if (run != LA_OK) {
+        cudaStreamSynchronize(cs);
+        return run;
     }
-    CK(cudaStreamSynchronize(st));
+    acc.ms_build = acc.ms_walk = -1.0;
     ctx->stats = acc;
+    ctx->extended = false;   // the device holds only the last chunk: nothing to replay
     out->n_ends = nE;
     out->ext_off = h_off;
     out->ext_seq = (const char *)ctx->h_ext_seq.p;
@@ -1041,6 +1108,40 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
     return LA_OK;
 }
 extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, false); }
+
+// Build-only replay (SURVEY §8(d) timing protocol step 5): the table-class kernels rerun, over the
+// class lists of the last la_extend, exactly the (end, k) attempts it made (k_start + i * shift for
+// i < n_attempts, the direction recorded per end in out_dir) with the link pass and the walk
+// disabled: staging, per-read prefix, table clear, filter and build passes (Alg 1) only.
+extern "C" la_status la_replay_build(la_ctx *ctx) {
+    if (!ctx) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
+    if (!ctx->extended) return fail(ctx, LA_ERR_STATE, "la_replay_build needs a completed la_extend of the loaded batch");
+    CK(cudaSetDevice(ctx->device));
+    cudaStream_t st = ctx->stream;
+    int *d_ctr = P<int>(ctx->ctrs);
+    unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
+    CK(cudaMemsetAsync(d_ctr + 15, 0, 4 * 8, st));   // overflow count + the class work counters
+    CK(cudaMemsetAsync(d_gst + 8, 0, 8 * GSTATS_WORDS * (N_SMEM_CLASSES + 1), st));
+    CK(cudaEventRecord(ctx->ev_rep[0], st));
+    const la_status s = launch_classes(ctx, true);
+    if (s != LA_OK) return s;
+    CK(cudaEventRecord(ctx->ev_rep[1], st));
+    int64_t *h64 = (int64_t *)ctx->h_small.p;
+    CK(cudaMemcpyAsync(h64, d_gst + 8, 8 * GSTATS_WORDS * (N_SMEM_CLASSES + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    float ms = 0;
+    cudaEventElapsedTime(&ms, ctx->ev_rep[0], ctx->ev_rep[1]);
+    ctx->stats.ms_build = ms;
+    ctx->stats.ms_walk = ctx->stats.ms_smem - ms;   // the rest of the table phase: link + walk + hand-offs
+    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
+        float m = 0;
+        cudaEventElapsedTime(&m, ctx->ev_cls0[c], ctx->ev_cls[c]);
+        ctx->stats.cls_build_ms[c] = m;
+        ctx->stats.cls_build_inserts[c] = h64[GSTATS_WORDS * c];
+    }
+    return LA_OK;
+}
 
 // ---- NEXT N1: on-device append of extensions to contigs (Fig 4 "Append extensions to contigs",
 // P:L464 "appended to the end of contig") -------------------------------------------------------

@@ -79,63 +79,67 @@ def select_contigs(batch, contig_ids):
     return out
 
 
-def gather_results(res: Result, contig_ids: np.ndarray, n_contigs_total: int, group=None, device=None):
-    """Gather every rank's Result to rank 0 and scatter it back into global end order.
+def _ranges(starts, lens):
+    """Concatenation of arange(starts[i], starts[i] + lens[i]) (vectorised)."""
+    lens = np.asarray(lens, np.int64)
+    tot = int(lens.sum())
+    if tot == 0:
+        return np.zeros(0, np.int64)
+    base = np.repeat(np.asarray(starts, np.int64) - np.concatenate([[0], np.cumsum(lens)[:-1]]), lens)
+    return base + np.arange(tot, dtype=np.int64)
 
-    One all_gather of the per-rank sizes, then one gather per packed array (the only inter-GPU
-    traffic, after extension).  Returns the merged Result on rank 0, None elsewhere."""
-    import torch
-    import torch.distributed as dist
-    rank, world = dist.get_rank(group), dist.get_world_size(group)
-    dev = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
-                                             if dist.get_backend(group) == "nccl" else torch.device("cpu"))
-    n_ends = 2 * int(contig_ids.shape[0])
-    lens = np.diff(res.ext_off).astype(np.int64)
-    meta = np.concatenate([[n_ends, int(res.ext_off[-1])]]).astype(np.int64)
-    sizes = [torch.zeros(2, dtype=torch.int64, device=dev) for _ in range(world)]
-    dist.all_gather(sizes, torch.from_numpy(meta).to(dev), group=group)
-    sizes = [s.cpu().numpy() for s in sizes]
-    max_e = max(int(s[0]) for s in sizes)
-    max_b = max(int(s[1]) for s in sizes)
 
-    def pad(a, n, dtype):
-        t = torch.zeros(max(n, 1), dtype=dtype, device=dev)
-        if a.shape[0]:
-            t[:a.shape[0]] = torch.from_numpy(np.ascontiguousarray(a)).to(dev)
-        return t
-
-    ids = np.stack([2 * contig_ids, 2 * contig_ids + 1], 1).reshape(-1)
-    packed = {
-        "ids": pad(ids, max_e, torch.int64),
-        "lens": pad(lens, max_e, torch.int64),
-        "codes": pad(np.stack([res.term, res.k_used, res.n_attempts], 1).reshape(-1).astype(np.uint8), 3 * max_e,
-                     torch.uint8),
-        "seq": pad(res.ext_seq, max_b, torch.uint8),
-    }
-    out = {}
-    for name, t in packed.items():
-        lst = [torch.empty_like(t) for _ in range(world)] if rank == 0 else None
-        dist.gather(t, lst, dst=0, group=group)
-        out[name] = [x.cpu().numpy() for x in lst] if rank == 0 else None
-    if rank != 0:
-        return None
+def merge_results(parts, n_contigs_total: int) -> Result:
+    """Scatter per-rank packed results into global end order (vectorised, no per-end loop).
+    parts: list of (end_ids int64[ne], lens int64[ne], codes uint8[ne, 3], seq uint8[nb])."""
     N = 2 * n_contigs_total
     glen = np.zeros(N, np.int64)
     term = np.zeros(N, np.uint8)
     k = np.zeros(N, np.uint8)
     att = np.zeros(N, np.uint8)
-    pieces = [None] * N
-    for r in range(world):
-        ne, nb = int(sizes[r][0]), int(sizes[r][1])
-        ids_r = out["ids"][r][:ne]
-        lens_r = out["lens"][r][:ne]
-        codes = out["codes"][r][:3 * ne].reshape(-1, 3) if ne else np.zeros((0, 3), np.uint8)
-        seq = out["seq"][r][:nb]
-        offs = np.concatenate([[0], np.cumsum(lens_r)])
-        glen[ids_r] = lens_r
-        term[ids_r], k[ids_r], att[ids_r] = codes[:, 0], codes[:, 1], codes[:, 2]
-        for i, e in enumerate(ids_r):
-            pieces[e] = seq[offs[i]:offs[i + 1]]
+    for ids, lens, codes, _ in parts:
+        glen[ids] = lens
+        term[ids], k[ids], att[ids] = codes[:, 0], codes[:, 1], codes[:, 2]
     ext_off = np.concatenate([[0], np.cumsum(glen)]).astype(np.int64)
-    ext_seq = np.concatenate([p for p in pieces if p is not None]) if N else np.zeros(0, np.uint8)
-    return Result(ext_off, ext_seq.astype(np.uint8), term, k, att)
+    ext_seq = np.zeros(int(ext_off[-1]), np.uint8)
+    for ids, lens, _, seq in parts:
+        if seq.shape[0]:
+            ext_seq[_ranges(ext_off[ids], lens)] = seq
+    return Result(ext_off, ext_seq, term, k, att)
+
+
+def gather_results(res: Result, contig_ids: np.ndarray, n_contigs_total: int, group=None, device=None):
+    """Gather every rank's Result to rank 0 and scatter it back into global end order.
+
+    One all_gather of the per-rank sizes, then exact-size point-to-point transfers of the packed
+    arrays to rank 0 (the only inter-GPU traffic, after extension; no padding to the largest rank),
+    merged without a per-end loop.  Returns the merged Result on rank 0, None elsewhere."""
+    import torch
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    dev = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
+                                             if dist.get_backend(group) == "nccl" else torch.device("cpu"))
+    contig_ids = np.asarray(contig_ids, np.int64)
+    ids = np.stack([2 * contig_ids, 2 * contig_ids + 1], 1).reshape(-1)
+    lens = np.diff(res.ext_off).astype(np.int64)
+    codes = np.stack([res.term, res.k_used, res.n_attempts], 1).astype(np.uint8).reshape(-1, 3)
+    meta = torch.tensor([ids.shape[0], int(res.ext_off[-1])], dtype=torch.int64, device=dev)
+    sizes = [torch.zeros(2, dtype=torch.int64, device=dev) for _ in range(world)]
+    dist.all_gather(sizes, meta, group=group)
+    sizes = [s.cpu().numpy() for s in sizes]
+    if rank != 0:
+        for a in (ids, lens, codes.reshape(-1), np.asarray(res.ext_seq, np.uint8)):
+            if a.shape[0]:
+                dist.send(torch.from_numpy(np.ascontiguousarray(a)).to(dev), dst=0, group=group)
+        return None
+    parts = [(ids, lens, codes, np.asarray(res.ext_seq, np.uint8))]
+    for r in range(1, world):
+        ne, nb = int(sizes[r][0]), int(sizes[r][1])
+        got = []
+        for n, dt in ((ne, torch.int64), (ne, torch.int64), (3 * ne, torch.uint8), (nb, torch.uint8)):
+            t = torch.empty(n, dtype=dt, device=dev)
+            if n:
+                dist.recv(t, src=r, group=group)
+            got.append(t.cpu().numpy())
+        parts.append((got[0], got[1], got[2].reshape(-1, 3), got[3]))
+    return merge_results(parts, n_contigs_total)

@@ -64,3 +64,29 @@ def test_append_extensions_null_context(lib):
     lib.la_append_extensions.argtypes = [ctypes.c_void_p, ctypes.c_int32] + [ctypes.c_void_p] * 6
     lib.la_append_extensions.restype = ctypes.c_int
     assert lib.la_append_extensions(None, 0, None, None, None, None, None, None) == -1
+
+
+def test_c_client_builds_and_links(lib):
+    """examples/abi_client.c is a plain C99 client of include/locassm.h: it compiles against the header
+    alone and its binary resolves liblocassm.so (it is run against a GPU in test_gpu_parity.py)."""
+    import subprocess
+    import sys
+    sys.path.insert(0, ROOT)
+    import __graft_entry__
+    __graft_entry__.build()
+    exe = os.path.join(ROOT, "examples", "abi_client")
+    assert os.path.exists(exe)
+    out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
+    assert "liblocassm.so" in out and "not found" not in out
+
+
+def test_api_rejects_wrong_dtypes(lib):
+    """The binding refuses arrays the C library would misread (int32 offsets, non-byte sequences)."""
+    import numpy as np
+    from gen import cases as C  # noqa: F401  (input layout only)
+    from paper_conf_sc_awanhedbdoy21_b200.api import _ptr_and_mem
+    with pytest.raises(ValueError):
+        _ptr_and_mem(np.zeros(3, np.int32), "read_off", "int64")
+    with pytest.raises(ValueError):
+        _ptr_and_mem(np.zeros(3, np.int64), "read_seq", "bytes")
+    assert _ptr_and_mem(np.zeros(3, np.int64), "read_off", "int64")[1] is False

@@ -311,3 +311,36 @@ def test_append_extensions_alignments(LA, seed):
     eoff = torch.from_numpy(pe + np.concatenate([[0], np.cumsum([len(x) for x in ext])])).cuda()
     seq, off = LA.append_extensions(cseq, coff, eoff, eseq)
     assert _appended_strings(seq, off) == oracle.append_extensions(contigs, ext)
+
+
+@pytest.mark.parametrize("cls", range(6))
+def test_class_by_key_format_matrix(LA, orc, cls):
+    """Every table class (0-4 shared memory, 5 = XL in global scratch) with inline keys (k <= 63) and
+    pointer keys (k >= 64), each forced (LA_FORCE_CLASS) and compared with the oracle end by end."""
+    b = cached_batch("C2", scale=0.03).select_contigs(np.arange(400))
+    for P, key in ((P0, "cls_inl_attempts"), (Params(k_start=65, k_min=57, k_max=97), "cls_ref_attempts")):
+        _, st = check(LA, orc, b, P, env={"LA_FORCE_CLASS": str(cls)})
+        assert st[key][cls] > 0, (cls, key, st[key])
+
+
+def test_replay_build_reruns_the_attempts(LA, orc):
+    """la_replay_build reruns exactly the extension's table builds (same inserts) and leaves its
+    results unchanged; attempts_hist counts every end."""
+    b = cached_batch("C2", scale=0.03)
+    r, st = check(LA, orc, b, P0)
+    rp = LA.replay_build()
+    assert sum(rp["cls_build_inserts"]) == st["inserts_smem"]
+    assert rp["ms_build"] > 0 and rp["ms_walk"] == pytest.approx(st["ms_smem"] - rp["ms_build"])
+    assert sum(st["attempts_hist"]) == b.n_ends
+    assert st["attempts_hist"] == np.bincount(np.minimum(r.n_attempts, 15), minlength=16).tolist()
+    r2 = LA.extend()
+    assert r2.ext_list() == r.ext_list() and np.array_equal(r2.term, r.term)
+
+
+def test_c_abi_client():
+    """The plain C client (examples/abi_client.c) on the device: closed-form pin P2 through the ABI."""
+    import subprocess
+    exe = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "examples", "abi_client")
+    out = subprocess.run([exe], capture_output=True, text=True, timeout=120)
+    assert out.returncode == 0, out.stderr
+    assert "abi_client ok" in out.stdout

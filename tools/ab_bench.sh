@@ -5,9 +5,8 @@ set -e
 # then: gpurun -- bash tools/ab_bench.sh
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -shared -Xcompiler -fPIC -I_headcsrc/include -o /tmp/head.so _headcsrc/csrc/locassm.cu
-nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -shared -Xcompiler -fPIC -Iinclude -DLA_CLAIM_PTX=1 -o /tmp/ptx.so paper_conf_sc_awanhedbdoy21_b200/csrc/locassm.cu
 for rep in 1 2; do
-for v in head new ptx; do
-  so=""; [ $v = head ] && so=/tmp/head.so; [ $v = ptx ] && so=/tmp/ptx.so
+for v in head new; do
+  so=""; [ $v = head ] && so=/tmp/head.so
   LA_SO=$so timeout 600 python bench.py --steps 3 --warmup 2 --no-cpu-baseline --no-e2e 2>/dev/null | python -c "import json,sys; d=json.load(sys.stdin); print('$v', d['ms_per_step'])"
 done; done
