@@ -128,6 +128,8 @@ typedef struct {
     /* per class: attempts built with inline keys (k <= 63) and with pointer keys (k >= 64) */
     int64_t cls_inl_attempts[6], cls_ref_attempts[6];
     int64_t attempts_hist[LA_HIST]; /* ends by number of attempts (last bin: >= LA_HIST-1)       */
+    int64_t cls_dead0[6];   /* per class: attempts decided after the filter pass (the start k-mer has
+                               < 2 voting occurrences: DEADEND at step 0 without building the table) */
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);

@@ -55,7 +55,7 @@ class la_stats(ctypes.Structure):
                 ("ms_build", ctypes.c_double), ("ms_walk", ctypes.c_double),
                 ("cls_build_ms", ctypes.c_double * 6), ("cls_build_inserts", ctypes.c_int64 * 6),
                 ("cls_inl_attempts", ctypes.c_int64 * 6), ("cls_ref_attempts", ctypes.c_int64 * 6),
-                ("attempts_hist", ctypes.c_int64 * LA_HIST)]
+                ("attempts_hist", ctypes.c_int64 * LA_HIST), ("cls_dead0", ctypes.c_int64 * 6)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",

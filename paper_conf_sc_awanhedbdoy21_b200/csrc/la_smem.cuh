@@ -45,6 +45,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_FQUEUE
 #define LA_FQUEUE 0   // 1: filtered builds keep per-position filter indices and queue survivors (r02 experiment)
 #endif
+#ifndef LA_DEAD0
+#define LA_DEAD0 1   // decide attempts whose start k-mer fails the filter without building (inl32_build_link)
+#endif
 #ifndef LA_MAX_LOAD
 #define LA_MAX_LOAD 0.70f
 #endif
@@ -295,10 +298,11 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
 constexpr uint32_t NEXT_NONE = 0x0FFFFFFFu;   // info word: next slot (28 bits) << 4 | visited << 3 | code
 
 struct GlobalStats {
-    // filtered: attempts built with the filter; inl / ref: attempts with inline / pointer (REF) keys
-    unsigned long long inserts, steps, attempts, filtered, inl, ref;
+    // filtered: attempts built with the filter; inl / ref: attempts with inline / pointer (REF) keys;
+    // dead0: attempts decided after the filter pass (start k-mer fails the filter: no build, no link)
+    unsigned long long inserts, steps, attempts, filtered, inl, ref, dead0;
 };
-constexpr int GSTATS_WORDS = 6;
+constexpr int GSTATS_WORDS = 7;
 // out_dir[e]: direction of the end's k shifts (-1 down, +1 up, 0 none) recorded by the extension,
 // so that la_replay_build can rerun exactly the same (end, k) attempts; OVF_DIR: the end left the
 // class kernel (table overflow -> global path) and is not replayed.
@@ -581,6 +585,8 @@ struct BuildCtl {           // builders' shared scratch
     int skip;               // 1: the current slot has no work (retired)
     int overflow, nclaim;
     uint32_t start;
+    uint32_t start_h;       // hash of the start k-mer (inline keys); start_ok: it has no N
+    int start_ok, dead0;    // dead0: the attempt is decided before the build (start k-mer < 2 votes)
     int lmin, lmax;
     uint32_t wsum[32];      // per builder warp: prefix-scan totals
 };
@@ -692,6 +698,23 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     T.cap = TC.cap;
     const uint32_t *R32 = (const uint32_t *)TC.rseq, *Q32 = (const uint32_t *)rqc;
     const int SW2 = 2 * TC.SW;
+    // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
+    K32<NW> Kst;
+    if (bt == 0) {
+        const int p = Tn - k;
+        bool hasN = false;
+        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
+        uint32_t Tw[2 * TAIL_W];
+#pragma unroll
+        for (int i = 0; i < TAIL_W; ++i) {
+            const uint64_t x = tail_e[i];
+            Tw[2 * i] = (uint32_t)x;
+            Tw[2 * i + 1] = (uint32_t)(x >> 32);
+        }
+        Kst = extract32<NW>(Tw, p, kmask32<NW>(k));
+        B.start_h = hash32<NW>(Kst);
+        B.start_ok = !hasN;
+    }
     if (!mbits || !LA_FQUEUE) {
         if (mbits) {
             // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
@@ -712,6 +735,22 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                      }
                                  });
             builders_sync(NB);
+            // The filter has no false negatives: a start k-mer whose B2 bit is clear has < 2 voting
+            // occurrences, so with V >= 2 (filters are only used then) it extends to DEADEND at step 0
+            // whatever the table holds (reading #1) — the walk of this attempt is decided: skip the
+            // build and the link pass (the attempt still counts its U inserts, the method's work).
+            if (LA_DEAD0) {
+                const uint32_t fs = filt32(B.start_h, mbits);
+                if (!B.start_ok || !((B2[fs >> 5] >> (fs & 31)) & 1u)) {
+                    if (bt == 0) {
+                        B.start = NONE;
+                        B.dead0 = 1;
+                    }
+                    builders_sync(NB);
+                    t_filter = t_build = la_clock();
+                    return;
+                }
+            }
         }
         t_filter = la_clock();
         // ---- build (Alg 1): every voting occurrence that passed the filter ----
@@ -809,26 +848,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         const uint32_t t = warp_lookup32<GT>(T, has && code < 4, key_form<NW>(K, h), h);
         if (has) info[s] = link_info(code, t);
     }
-    if (bt == 0) {
-        // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
-        const int p = Tn - k;
-        bool hasN = false;
-        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
-        uint32_t st = NONE;
-        if (!hasN) {
-            uint32_t Tw[2 * TAIL_W];
-#pragma unroll
-            for (int i = 0; i < TAIL_W; ++i) {
-                const uint64_t x = tail_e[i];
-                Tw[2 * i] = (uint32_t)x;
-                Tw[2 * i + 1] = (uint32_t)(x >> 32);
-            }
-            const K32<NW> K = extract32<NW>(Tw, p, kmask32<NW>(k));
-            const uint32_t h = hash32<NW>(K);
-            st = lookup32<GT>(T, key_form<NW>(K, h), h);
-        }
-        B.start = st;
-    }
+    if (bt == 0) B.start = B.start_ok ? lookup32<GT>(T, key_form<NW>(Kst, B.start_h), B.start_h) : NONE;
 }
 
 template <bool INL, bool GT>
@@ -1086,6 +1106,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             B.skip = 0;
             B.overflow = 0;
             B.nclaim = 0;
+            B.dead0 = 0;
             if (E.done) {   // refill the slot with the next end, or retire it
                 int idx, e = 0;
                 do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
@@ -1260,6 +1281,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
                                       t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
+            if (bt == 0) s_acc[6] += B.dead0;
         }
         builders_sync(NB);   // info buffer complete; the table is free for the next build
         {
@@ -1290,6 +1312,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
         atomicAdd(&gstats->filtered, s_acc[3]);
         atomicAdd(&gstats->inl, s_acc[4]);
         atomicAdd(&gstats->ref, s_acc[5]);
+        atomicAdd(&gstats->dead0, s_acc[6]);
         if (prof)
             for (int i = 0; i < 6; ++i) atomicAdd(&prof[i], (unsigned long long)b_t[i]);
     }
@@ -1420,6 +1443,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             if (bt == 0) {
                 B.overflow = 0;
                 B.nclaim = 0;
+                B.dead0 = 0;
             }
             const long long tc = la_clock();
             {
@@ -1448,6 +1472,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             b_t[3] += t_filter - td;
             b_t[4] += t_build - t_filter;
             b_t[5] += te - t_build;
+            if (bt == 0) s_acc[6] += B.dead0;
             if (B.overflow) {
                 ovf = true;
                 break;

@@ -72,6 +72,11 @@ const ClassEntry kClassKernels[] = {   // the five classes la_create configures 
     {256, 3, false, k_smem<256, false, 3>},
     {512, 2, false, k_smem<512, false, 2>},
     {1024, 1, false, k_smem<1024, false, 1>},
+#ifdef LA_EXTRA_CLASSES   // tuning builds only (tools/ab_build.sh): other (threads x CTAs/SM) shapes
+    {64, 16, true, k_small<64, 16>},   {128, 8, true, k_small<128, 8>},  {96, 8, true, k_small<96, 8>},
+    {256, 4, false, k_smem<256, false, 4>}, {256, 3, true, k_small<256, 3>}, {32, 24, true, k_small<32, 24>},
+    {32, 16, true, k_small<32, 16>},   {64, 10, true, k_small<64, 10>},
+#endif
 };
 const ClassEntry *find_class_kernel(int threads, int ctas, bool small) {
     for (const ClassEntry &k : kClassKernels)
@@ -830,6 +835,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         ctx->stats.cls_filtered[c] = g[3];
         ctx->stats.cls_inl_attempts[c] = g[4];
         ctx->stats.cls_ref_attempts[c] = g[5];
+        ctx->stats.cls_dead0[c] = g[6];
         h64[1] += g[0];
         h64[2] += g[1];
         h64[3] += g[2];
@@ -1083,6 +1089,7 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
                 acc.cls_filtered[q] += x.cls_filtered[q];
                 acc.cls_inl_attempts[q] += x.cls_inl_attempts[q];
                 acc.cls_ref_attempts[q] += x.cls_ref_attempts[q];
+                acc.cls_dead0[q] += x.cls_dead0[q];
                 acc.cls_ms[q] += x.cls_ms[q];
             }
             for (int q = 0; q < LA_HIST; ++q) acc.attempts_hist[q] += x.attempts_hist[q];

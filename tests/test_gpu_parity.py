@@ -340,7 +340,12 @@ def test_replay_build_reruns_the_attempts(LA, orc):
 def test_c_abi_client():
     """The plain C client (examples/abi_client.c) on the device: closed-form pin P2 through the ABI."""
     import subprocess
-    exe = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "examples", "abi_client")
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import __graft_entry__
+    __graft_entry__.build()   # (re)builds the client against the current header and library
+    exe = os.path.join(root, "examples", "abi_client")
     out = subprocess.run([exe], capture_output=True, text=True, timeout=120)
     assert out.returncode == 0, out.stderr
     assert "abi_client ok" in out.stdout
