@@ -96,9 +96,10 @@ int main(void) {
     CHECK(r.k_used[1] == 33 && r.n_attempts[1] == (33 - 21) / 8 + 1, "k_used %d attempts %d", r.k_used[1],
           r.n_attempts[1]);
     CHECK(st.ext_bases == want_len, "stats.ext_bases %lld", (long long)st.ext_bases);
-    CHECK(la_destroy(ctx) == LA_OK, "la_destroy");
+    /* results are library-owned: read them before la_destroy */
     printf("abi_client ok: right extension %lld bases (closed form %d), DEADEND, k %d, %d attempts\n",
            (long long)got_len, want_len, r.k_used[1], r.n_attempts[1]);
+    CHECK(la_destroy(ctx) == LA_OK, "la_destroy");
     free(rseq);
     free(rqual);
     free(roff);

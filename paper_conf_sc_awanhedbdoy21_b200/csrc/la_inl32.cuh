@@ -192,6 +192,27 @@ __device__ __forceinline__ void vote32(const Tab32 &T, uint32_t s, uint32_t b, b
         if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;
     }
 }
+// Same vote with the carry check of the PREVIOUS vote of this lane (pend: its old counter word shifted
+// to the voted field): the atomic's return value is first used one insert later, so the warp does not
+// wait for the shared-memory atomic's round trip on every insert.  flush_vote32 checks the last one.
+#ifndef LA_DEFER_VOTE
+#define LA_DEFER_VOTE 1
+#endif
+template <bool GT>
+__device__ __forceinline__ void vote32d(const Tab32 &T, uint32_t s, uint32_t b, bool hi, volatile int *ovf,
+                                        uint32_t &pend) {
+    if (GT || LA_ABL_NOVOTE || !LA_DEFER_VOTE) {
+        vote32<GT>(T, s, b, hi, ovf);
+        return;
+    }
+    if ((pend & 0xffu) == 0xffu) *ovf = 1;
+    pend = atomicAdd(&T.c32[2 * s + (hi ? 1u : 0u)], 1u << (8 * b)) >> (8 * b);
+}
+__device__ __forceinline__ void flush_vote32(uint32_t &pend, volatile int *ovf) {
+    if ((pend & 0xffu) == 0xffu) *ovf = 1;
+    pend = 0;
+}
+
 template <bool GT>
 __device__ __forceinline__ void votes32(const Tab32 &T, uint32_t s, uint32_t lo[4], uint32_t hi[4]) {
     if (GT) {
@@ -225,7 +246,8 @@ __device__ __forceinline__ int cmp_slot(const Tab32 &T, uint32_t s, uint4 v, con
 // claims are appended to the claim list once per warp (ballot + one atomic).
 template <bool GT>
 __device__ __forceinline__ void warp_insert32(const Tab32 &T, bool want, const uint4 f, uint32_t h, uint32_t nb,
-                                              bool hi, int lane, int *nclaim, int claim_limit, volatile int *ovf) {
+                                              bool hi, int lane, int *nclaim, int claim_limit, volatile int *ovf,
+                                              uint32_t &vpend) {
     uint32_t s = slot32(h, T.cap), hit = 0;
     bool pend = want, found = false;
     while (__any_sync(0xffffffffu, pend)) {
@@ -280,7 +302,7 @@ __device__ __forceinline__ void warp_insert32(const Tab32 &T, bool want, const u
             T.list[idx] = (uint16_t)hit;
         }
     }
-    if (found) vote32<GT>(T, hit, nb, hi, ovf);
+    if (found) vote32d<GT>(T, hit, nb, hi, ovf, vpend);
 }
 
 // Convergent lookup (no insert): slot of the key or NONE
@@ -336,7 +358,7 @@ __device__ __forceinline__ uint32_t nmask32(uint32_t q) { return q & (q >> 1) & 
 // ulen, so the (read, offset) of a position is one multiply-high (no prefix walk).
 // f(inr, act, g, K, h, nb, hi): inr = this lane has a position g this iteration; act = it is a voting
 // occurrence (q >= q_lo, no N in the window and in the following base).
-template <int NW, typename F>
+template <int NW, int UNR = 1, typename F>
 __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rseq, const uint32_t *__restrict__ rqc,
                                                  const uint8_t *__restrict__ rflag, const uint32_t *pref,
                                                  long long r0, int r, int SW2, int k, int ulen, int wid, int nwarps,
@@ -361,6 +383,38 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
         j = lo;
         pj0 = pref[j];
         pj1 = pref[j + 1];
+    }
+    // UNR > 1 (uniform read lengths only): a lane takes positions g, g+32, ... per iteration, so the
+    // independent load -> hash -> filter chains of UNR positions overlap (the filter pass)
+    if (UNR > 1 && ulen > 0) {
+        for (uint32_t base = wb; base < we; base += 32u * UNR, g += 32u * UNR) {
+#pragma unroll
+            for (int u = 0; u < UNR; ++u) {
+                const uint32_t gu = g + 32u * u;
+                const bool act = gu < we;
+                uint32_t jj = __umulhi(gu, magic);
+                uint32_t pp = gu - jj * np;
+                if (pp >= np) { ++jj; pp -= np; }
+                const int p = act ? (int)pp : 0;
+                const long long row = (r0 + (act ? (int)jj : 0)) * (long long)SW2;
+                const uint32_t *R = rseq + row, *Q = rqc + row;
+                const K32<NW> K = extract32<NW>(R, p, m);
+                const uint32_t nb = base32(R, p + k), nq = base32(Q, p + k);
+                bool vote = act && (nq - 1u < 2u);
+                if (vote && rflag[r0 + jj]) {
+                    const int q = p >> 4, s = (p & 15) << 1;
+                    uint32_t any = 0;
+#pragma unroll
+                    for (int w = 0; w < NW; ++w) {
+                        const uint32_t mw = w == NW - 1 ? m.m1 : (w == NW - 2 ? m.m2 : ~0u);
+                        any |= __funnelshift_l(nmask32(rw32(Q, q + w + 1)), nmask32(rw32(Q, q + w)), s) & mw;
+                    }
+                    if (any) vote = false;
+                }
+                f(act, vote, gu, K, hash32<NW>(K), nb, nq == 2u);
+            }
+        }
+        return;
     }
     for (uint32_t base = wb; base < we; base += 32u, g += 32u) {
         if (((base - wb) & 127u) == 0 && __shfl_sync(0xffffffffu, *stop, 0)) return;   // every 4th iteration

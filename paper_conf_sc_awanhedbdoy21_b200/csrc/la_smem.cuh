@@ -45,6 +45,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_FQUEUE
 #define LA_FQUEUE 0   // 1: filtered builds keep per-position filter indices and queue survivors (r02 experiment)
 #endif
+#ifndef LA_FILTER_UNROLL
+#define LA_FILTER_UNROLL 2   // positions per lane per iteration of the filter pass (la_inl32.cuh)
+#endif
 #ifndef LA_DEAD0
 #define LA_DEAD0 1   // decide attempts whose start k-mer fails the filter without building (inl32_build_link)
 #endif
@@ -718,7 +721,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     if (!mbits || !LA_FQUEUE) {
         if (mbits) {
             // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
-            warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
+            warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
                                  [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
                                      if (!act) return;
                                      const uint32_t fi = filt32(h, mbits);
@@ -754,6 +757,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         }
         t_filter = la_clock();
         // ---- build (Alg 1): every voting occurrence that passed the filter ----
+        uint32_t pend = 0;   // carry check of this lane's last vote (vote32d)
         warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
                              [&](bool, bool act, uint32_t, const K32<NW> &K, uint32_t h, uint32_t nb, bool hi) {
                                  bool want = act;
@@ -762,8 +766,9 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                      want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
                                  }
                                  warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim,
-                                                   claim_limit, &B.overflow);
+                                                   claim_limit, &B.overflow, pend);
                              });
+        flush_vote32(pend, &B.overflow);
     } else {
         // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4); every position's
         // filter bit index (or FNONE: no vote) is kept for the build pass ----
@@ -789,6 +794,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         const uint32_t total = pref[r];
         const uint32_t wb = (uint32_t)(((uint64_t)total * (uint32_t)wid) / (uint32_t)nwarps);
         const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
+        uint32_t pend = 0;   // carry check of this lane's last vote (vote32d)
         auto insert_batch = [&](bool has, uint32_t g) {
             int j = 0, p = 0;
             if (has) pos_of(g, pref, r, ulen, k, j, p);
@@ -797,7 +803,8 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
             const K32<NW> K = extract32<NW>(Rr, p, m);
             const uint32_t nb = base32(Rr, p + k), nq = base32(Qr, p + k);
             const uint32_t h = hash32<NW>(K);
-            warp_insert32<GT>(T, has, key_form<NW>(K, h), h, nb, nq == 2u, lane, &B.nclaim, claim_limit, &B.overflow);
+            warp_insert32<GT>(T, has, key_form<NW>(K, h), h, nb, nq == 2u, lane, &B.nclaim, claim_limit, &B.overflow,
+                              pend);
         };
         uint32_t qn = 0;   // queued positions (warp-uniform)
         const unsigned lt = (1u << lane) - 1u;
@@ -823,6 +830,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         }
         __syncwarp();
         if (__shfl_sync(0xffffffffu, *stop, 0) == 0 && qn) insert_batch(lane < qn, lane < qn ? queue[lane] : 0u);
+        flush_vote32(pend, &B.overflow);
     }
     builders_sync(NB);
     t_build = la_clock();
