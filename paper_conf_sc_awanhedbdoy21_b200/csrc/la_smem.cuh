@@ -1004,13 +1004,20 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             if (lane == 0) mbar_wait(&built[s], (phase >> s) & 1u);
             w_wait += la_clock() - tw0;
             phase ^= 1u << s;
-            __syncwarp();
             EndSlot &E = S[s];
-            if (E.dead) {
+            // lane 0 alone reads the slot's state (it waited on the mbarrier) and broadcasts it
+            int st_dead = 0, st_ovf = 0;
+            if (lane == 0) {
+                st_dead = E.dead;
+                st_ovf = E.ovf;
+            }
+            st_dead = __shfl_sync(0xffffffffu, st_dead, 0);
+            st_ovf = __shfl_sync(0xffffffffu, st_ovf, 0);
+            if (st_dead) {
                 alive &= ~(1u << s);
                 continue;
             }
-            if (E.ovf) {   // the build overflowed: the global path owns this end; pass the slot back
+            if (st_ovf) {   // the build overflowed: the global path owns this end; pass the slot back
                 if (lane == 0) mbar_arrive(&walked[s]);
                 continue;
             }
@@ -1066,7 +1073,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 }
             } else if (done) {
                 // ---- the selected walk -> HBM ----
-                const int e = E.e;
+                __syncwarp();   // lane 0's walk string is complete
+                const int e = __shfl_sync(0xffffffffu, lane == 0 ? E.e : 0, 0);
                 const uint8_t *bw = wstr + (2 * s + bb) * Wp;
                 uint8_t *dst = walk_buf + (size_t)e * P.W;
                 for (int i = lane; i < bl; i += 32) dst[i] = bw[i];
@@ -1111,7 +1119,6 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 wphase ^= 1u << s;
             }
             first &= ~(1u << s);
-            B.skip = 0;
             B.overflow = 0;
             B.nclaim = 0;
             B.dead0 = 0;
@@ -1123,7 +1130,6 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
                 if (idx >= n_list) {
                     E.dead = 1;
-                    B.skip = 1;
                     mbar_arrive(&built[s]);   // the walker sees `dead` and retires the slot too
                 } else {
                     E.e = e;
@@ -1152,7 +1158,9 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
         builders_sync(NB);
         const long long tb = la_clock();
         b_t[0] += tb - ta;
-        if (B.skip) {
+        // the slot's own, monotonic `dead` flag — not the shared B.skip, which the leader rewrites for
+        // the other slot right away (a builder still reading B.skip could see the other slot's value)
+        if (E.dead) {
             alive &= ~(1u << s);
             continue;
         }
