@@ -129,6 +129,7 @@ struct Tab32 {
     uint32_t *c32;          // counters: per slot two u32 of four 8-bit fields (shared) / 8 x u32 (XL)
     uint16_t *list;         // claimed slots in claim order
     uint32_t cap;           // even
+    int wide;               // XL: 32-bit counter fields (else 16-bit)
 };
 
 template <bool GT>
@@ -179,6 +180,11 @@ __device__ __forceinline__ uint4 cas_slot(const Tab32 &T, uint32_t s, const uint
 // One vote for base b of slot s: high-tier (q >= q_hi) and low-only (q_lo <= q < q_hi)
 // votes in separate counter words; the low tier of reading #1 is their sum.  Shared memory: 8-bit
 // fields, a field about to carry flags the end for the global path (reading #15); XL: 8 x u32.
+// Counters.  Shared-memory tables: per slot two u32 of four 8-bit fields (low-only votes, high
+// votes); a field about to carry flags the end for the global path (reading #15).  XL tables (global
+// scratch, GT): no carry check (a global atomic's return trip is slow), fire-and-forget RED.ADD on
+// fields wide enough for the attempt: 16-bit fields (4 x u32 per slot) when the attempt has fewer than
+// 65536 voting occurrences (a field counts at most all of them), else 8 x u32 (`wide`).
 template <bool GT>
 __device__ __forceinline__ void vote32(const Tab32 &T, uint32_t s, uint32_t b, bool hi, volatile int *ovf) {
     if (LA_ABL_NOVOTE) {
@@ -186,7 +192,8 @@ __device__ __forceinline__ void vote32(const Tab32 &T, uint32_t s, uint32_t b, b
         return;
     }
     if (GT) {
-        atomicAdd(&T.c32[8 * (size_t)s + (hi ? 4u : 0u) + b], 1u);
+        if (T.wide) atomicAdd(&T.c32[8 * (size_t)s + (hi ? 4u : 0u) + b], 1u);
+        else atomicAdd(&T.c32[4 * (size_t)s + (hi ? 2u : 0u) + (b >> 1)], 1u << (16 * (b & 1u)));
     } else {
         const uint32_t old = atomicAdd(&T.c32[2 * s + (hi ? 1u : 0u)], 1u << (8 * b));
         if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;
@@ -215,10 +222,15 @@ __device__ __forceinline__ void flush_vote32(uint32_t &pend, volatile int *ovf) 
 
 template <bool GT>
 __device__ __forceinline__ void votes32(const Tab32 &T, uint32_t s, uint32_t lo[4], uint32_t hi[4]) {
-    if (GT) {
+    if (GT && T.wide) {
         const uint4 a = ((const uint4 *)T.c32)[2 * (size_t)s], c = ((const uint4 *)T.c32)[2 * (size_t)s + 1];
         hi[0] = c.x; hi[1] = c.y; hi[2] = c.z; hi[3] = c.w;
         lo[0] = a.x + c.x; lo[1] = a.y + c.y; lo[2] = a.z + c.z; lo[3] = a.w + c.w;
+    } else if (GT) {
+        const uint4 a = ((const uint4 *)T.c32)[s];
+        hi[0] = a.z & 0xffffu; hi[1] = a.z >> 16; hi[2] = a.w & 0xffffu; hi[3] = a.w >> 16;
+        lo[0] = (a.x & 0xffffu) + hi[0]; lo[1] = (a.x >> 16) + hi[1];
+        lo[2] = (a.y & 0xffffu) + hi[2]; lo[3] = (a.y >> 16) + hi[3];
     } else {
         const uint2 w = ((const uint2 *)T.c32)[s];
 #pragma unroll

@@ -132,15 +132,18 @@ __host__ __device__ __forceinline__ uint32_t fpos_bytes(uint32_t U, bool gt) {
 // the per-read position prefix array (pref_bytes(r)).
 // Counters: shared-memory tables pack lo[4] | hi[4] as 8-bit fields (8 B, carry detected); global
 // (XL) tables use 8 x u32 (32 B) updated with fire-and-forget RED.ADD.
-__host__ __device__ __forceinline__ uint32_t cnt_bytes(bool gt) { return gt ? 32u : 8u; }
+// counter bytes per slot: shared tables 8 (8-bit fields), XL 16 (16-bit fields) or 32 (wide, U >= 65536)
+__host__ __device__ __forceinline__ uint32_t cnt_bytes(bool gt, bool wide = false) { return gt ? (wide ? 32u : 16u) : 8u; }
+__host__ __device__ __forceinline__ bool xl_wide(uint32_t U) { return U >= 65536u; }
 
 __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_t U, bool allow_filter,
                                                      uint32_t kbytes, int r, bool gt, int SW) {
+    const bool wide = gt && xl_wide(U);
     SmemTab T;
     const uint32_t sb = gt ? 0u : stage_bytes(r, SW);   // shared-memory tables: reads staged first
     const uint32_t pb = pref_bytes(r) + sb;
     const uint32_t tab = F.tab_bytes > pb ? F.tab_bytes - pb : 0u;
-    const uint32_t per_slot = kbytes + cnt_bytes(gt) + 2u;   // key + counters + claim-list entry (u16)
+    const uint32_t per_slot = kbytes + cnt_bytes(gt, wide) + 2u;   // key + counters + claim-list entry (u16)
     uint32_t cap_nf = tab / per_slot;
     if (cap_nf > F.icap) cap_nf = F.icap;
     cap_nf &= ~1u;
@@ -180,7 +183,7 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
     T.cap = cap;
     T.mwords = mwords;
     T.off_cnts = T.off_keys + cap * kbytes;
-    T.off_list = T.off_cnts + cap * cnt_bytes(gt);
+    T.off_list = T.off_cnts + cap * cnt_bytes(gt, wide);
     // shared: right after B2; XL: in the global scratch after the claim list
     T.off_f = gt ? ((T.off_list + cap * 2u + 15u) & ~15u) : (T.off_b2 + mwords * 4u);
     return T;
@@ -236,7 +239,7 @@ __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_
     uint32_t cap = xl_needed_cap(r_max, U_max, filter);
     if (cap < min_table_cap(XL_THREADS)) cap = min_table_cap(XL_THREADS);   // claims + in-flight < cap
     if (cap > icap) cap = icap;
-    return (pref_bytes((int)r_max) + 48u + cap * (16u + cnt_bytes(true) + 2u) + fpos_bytes((uint32_t)U_max, true) +
+    return (pref_bytes((int)r_max) + 48u + cap * (16u + cnt_bytes(true, true) + 2u) + fpos_bytes((uint32_t)U_max, true) +
             255u) & ~255u;
 }
 
@@ -359,6 +362,7 @@ struct TabCtx {   // what a table operation needs
     uint32_t cap;
     const uint64_t *rseq;   // packed reads (global), for REF-format key verification
     int SW, k, KW;
+    int wide;               // XL: 32-bit counter fields (U >= 65536), else 16-bit
 };
 
 // One vote for base b of slot s: a single atomic per vote.  Counter words hold the
@@ -367,8 +371,9 @@ struct TabCtx {   // what a table operation needs
 // a field about to carry flags the end for the global path; global (XL): 8 x u32, RED.ADD.
 template <bool GT>
 __device__ __forceinline__ void vote_add(const TabCtx &T, uint32_t s, uint32_t b, bool hi, volatile int *ovf) {
-    if (GT) {
-        atomicAdd(&T.c32[8 * (size_t)s + (hi ? 4u : 0u) + b], 1u);
+    if (GT) {   // XL: fire-and-forget RED.ADD on 16-bit or (wide) 32-bit fields, as vote32 (la_inl32.cuh)
+        if (T.wide) atomicAdd(&T.c32[8 * (size_t)s + (hi ? 4u : 0u) + b], 1u);
+        else atomicAdd(&T.c32[4 * (size_t)s + (hi ? 2u : 0u) + (b >> 1)], 1u << (16 * (b & 1u)));
     } else {
         const uint32_t old = atomicAdd(&T.c32[2 * s + (hi ? 1u : 0u)], 1u << (8 * b));
         if (((old >> (8 * b)) & 0xffu) == 0xffu) *ovf = 1;   // an 8-bit counter would carry
@@ -377,10 +382,15 @@ __device__ __forceinline__ void vote_add(const TabCtx &T, uint32_t s, uint32_t b
 
 template <bool GT>
 __device__ __forceinline__ void votes_of(const TabCtx &T, uint32_t s, uint32_t lo[4], uint32_t hi[4]) {
-    if (GT) {
+    if (GT && T.wide) {
         const uint4 a = ((const uint4 *)T.c32)[2 * (size_t)s], c = ((const uint4 *)T.c32)[2 * (size_t)s + 1];
         hi[0] = c.x; hi[1] = c.y; hi[2] = c.z; hi[3] = c.w;
         lo[0] = a.x + c.x; lo[1] = a.y + c.y; lo[2] = a.z + c.z; lo[3] = a.w + c.w;
+    } else if (GT) {
+        const uint4 a = ((const uint4 *)T.c32)[s];
+        hi[0] = a.z & 0xffffu; hi[1] = a.z >> 16; hi[2] = a.w & 0xffffu; hi[3] = a.w >> 16;
+        lo[0] = (a.x & 0xffffu) + hi[0]; lo[1] = (a.x >> 16) + hi[1];
+        lo[2] = (a.y & 0xffffu) + hi[2]; lo[3] = (a.y >> 16) + hi[3];
     } else {
         const uint2 w = ((const uint2 *)T.c32)[s];
 #pragma unroll
@@ -699,6 +709,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     T.c32 = TC.c32;
     T.list = TC.list;
     T.cap = TC.cap;
+    T.wide = TC.wide;
     const uint32_t *R32 = (const uint32_t *)TC.rseq, *Q32 = (const uint32_t *)rqc;
     const int SW2 = 2 * TC.SW;
     // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
@@ -1248,7 +1259,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             if (TB.cap > need) {
                 TB.cap = (need + 1u) & ~1u;
                 TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
-                TB.off_list = TB.off_cnts + TB.cap * cnt_bytes(true);
+                TB.off_list = TB.off_cnts + TB.cap * cnt_bytes(true, xl_wide(U));
                 TB.off_f = (TB.off_list + TB.cap * 2u + 15u) & ~15u;
             }
         }
@@ -1271,11 +1282,12 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             T.SW = SW;
             T.k = k;
             T.KW = KW;
+            T.wide = GT && xl_wide(U) ? 1 : 0;
             // clear keys + counters (contiguous) and the filters
             {
                 const uint4 z = make_uint4(0, 0, 0, 0);
                 uint4 *a = (uint4 *)T.keys;
-                const uint32_t n16 = (TB.cap * (key_bytes(k) + cnt_bytes(GT))) / 16u;
+                const uint32_t n16 = (TB.cap * (key_bytes(k) + cnt_bytes(GT, GT && xl_wide(U)))) / 16u;
                 for (uint32_t i = bt; i < n16; i += NB) a[i] = z;
                 for (uint32_t i = bt; i < 2u * TB.mwords; i += NB) B1[i] = 0;   // B1, B2 contiguous
             }
@@ -1456,6 +1468,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             T.SW = SW;
             T.k = k;
             T.KW = KW;
+            T.wide = 0;
             if (bt == 0) {
                 B.overflow = 0;
                 B.nclaim = 0;

@@ -349,3 +349,26 @@ def test_c_abi_client():
     out = subprocess.run([exe], capture_output=True, text=True, timeout=120)
     assert out.returncode == 0, out.stderr
     assert "abi_client ok" in out.stdout
+
+
+def test_xl_wide_counters(LA, orc):
+    """XL tables with 32-bit counter fields: an end with >= 65536 voting occurrences per attempt (700
+    reads of a 20,000x end of C3) forced into the XL class; and the same end's first 300 reads (16-bit
+    fields).  Both against the oracle."""
+    b = cached_batch("C3")
+    r = b.reads_per_end()
+    e = int(np.nonzero(r >= 10000)[0][0])
+    c = e // 2
+    contig = b.contig_seq[b.contig_off[c]:b.contig_off[c + 1]].tobytes().decode()
+
+    def reads(n):
+        out = []
+        for j in range(b.end_read_off[e], b.end_read_off[e] + n):
+            s0, s1 = b.read_off[j], b.read_off[j + 1]
+            out.append((b.read_seq[s0:s1].tobytes().decode(), b.read_qual[s0:s1].tobytes().decode()))
+        return out
+    for n in (700, 300):
+        ends = [[], reads(n)] if e % 2 else [reads(n), []]
+        sub = C.Batch.from_lists([contig], ends)
+        _, st = check(LA, orc, sub, P0, env={"LA_FORCE_CLASS": "5"})
+        assert st["cls_inl_attempts"][5] > 0 and st["ends_by_class"][4] == 0
