@@ -115,7 +115,8 @@ typedef struct {
     int64_t xl_scratch_bytes;
     /* per table class: 0..4 shared memory (64, 128, 256@3, 256@2, 512 threads), 5 = XL */
     int64_t cls_ends[6], cls_inserts[6], cls_attempts[6], cls_filtered[6];
-    double cls_ms[6];            /* start -> end of each class kernel (classes run concurrently)   */
+    double cls_ms[6];            /* device time of each class kernel (serial by default; spans if
+                                    LA_CONCURRENT_CLASSES=1 launches them together)                */
     /* LA_PROFILE=1 only: per class, summed clock64 cycles of the builders' leader (wait for the
        walker, prefix, clear, filter pass, build pass, link) and of the walker (wait, walk) */
     uint64_t prof_cycles[6][8];

@@ -122,10 +122,14 @@ struct la_ctx {
     cudaEvent_t ev_rep[2] = {};   // la_replay_build start / end
     cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] classes may start
     cudaEvent_t ev_cls0[N_SMEM_CLASSES + 1] = {};  // start of class c ([N] = XL)
-    // one stream per table class: the persistent class kernels are launched together (largest tables
+    // one stream per table class (LA_CONCURRENT_CLASSES=1): the persistent class kernels launched together (largest tables
     // first) so that the tail of one class overlaps the start of the next; LA_SERIAL_CLASSES=1: one stream
     cudaStream_t cls_stream[N_SMEM_CLASSES + 1] = {};
-    bool concurrent_classes = true;
+    // r02: the class kernels run one after another on the context stream by default.  Measured on C4S,
+    // launching them on six streams at once gave the same step time (each persistent class kernel
+    // fills the GPU, so only their tails can overlap) while making the per-class times overlapping
+    // spans; LA_CONCURRENT_CLASSES=1 restores the concurrent launch.
+    bool concurrent_classes = false;
     la_stats stats{};
 };
 
@@ -285,6 +289,7 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
     for (auto &e : ctx->ev_cls0) cudaEventCreate(&e);
     for (auto &q : ctx->cls_stream)
         if (cudaStreamCreateWithFlags(&q, cudaStreamNonBlocking) != cudaSuccess) q = nullptr;
+    if (getenv("LA_CONCURRENT_CLASSES") && atoi(getenv("LA_CONCURRENT_CLASSES"))) ctx->concurrent_classes = true;
     if (getenv("LA_SERIAL_CLASSES") && atoi(getenv("LA_SERIAL_CLASSES"))) ctx->concurrent_classes = false;
     bool attr_ok = cudaFuncSetAttribute(k_smem<XL_THREADS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         ctx->cls_bytes[N_SMEM_CLASSES - 1]) == cudaSuccess;
