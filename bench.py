@@ -370,6 +370,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-replay", action="store_true", help="skip the build-only replay (roofline_build)")
     ap.add_argument("--e2e-chunks", type=int, default=8)
+    ap.add_argument("--coexec-share", type=float, default=0.05,
+                    help="NEXT N3 measurement: share of the smallest class's ends on host threads (0: skip)")
+    ap.add_argument("--coexec-threads", type=int, default=0, help="host threads for N3 (0: cores - 2)")
     ap.add_argument("--k-start", type=int, default=None,
                     help="NEXT N2: LA at another k of the assembler's contig iteration (21, 33, 55, 77)")
     args = ap.parse_args()
@@ -457,6 +460,32 @@ def main():
             if i:
                 rms.append(la.stats())
         replay = rms
+
+    # ---------------- NEXT N3: CPU+GPU co-execution (outside the timed step) ----------------
+    n3 = None
+    if args.coexec_share > 0:
+        thr = args.coexec_threads or max(1, (os.cpu_count() or 2) - 2)
+        la.set_coexec(thr, args.coexec_share)
+        ms3 = []
+        for i in range(4):
+            with torch.cuda.stream(stream):
+                flush_l2(flush)
+                a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a0.record(stream)
+            la.extend_device()
+            a1.record(stream)
+            a1.synchronize()
+            if i:
+                ms3.append(a0.elapsed_time(a1))
+        st3 = la.stats()
+        la.set_coexec(0, 0.0)
+        m3 = statistics.median(ms3)
+        n3 = {"host_threads": thr, "share_of_smallest_class": args.coexec_share, "host_ends": st3["cpu_ends"],
+              "host_inserts": st3["cpu_inserts"], "ms_per_step": m3, "gpu_only_ms_per_step": ms_total / args.steps,
+              "value": st3["ext_bases"] / (m3 / 1e3), "unit": UNIT,
+              "note": "la_set_coexec: the lightest ends of the smallest class on host threads while the GPU "
+                      "runs (NEXT N3, paper §4.3); this rank, CUDA events around la_extend_device, outside "
+                      "the timed step; DESIGN.md §10c"}
 
     # ---------------- NEXT N1: on-device append of the extensions (not part of the step) ----------------
     d = la.extend_device()
@@ -586,6 +615,7 @@ def main():
         "gather_ms": gather_ms,
         "parity": parity,
         "append_n1": dict(append_n1, peak=peaks["hbm_gbs"], frac=append_n1["achieved"] / peaks["hbm_gbs"]),
+        "coexec_n3": n3,
         "paper": PAPER,
     }
     if cpu:

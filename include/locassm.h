@@ -131,6 +131,9 @@ typedef struct {
     int64_t attempts_hist[LA_HIST]; /* ends by number of attempts (last bin: >= LA_HIST-1)       */
     int64_t cls_dead0[6];   /* per class: attempts decided after the filter pass (the start k-mer has
                                < 2 voting occurrences: DEADEND at step 0 without building the table) */
+    /* NEXT N3 co-execution (la_set_coexec): ends extended on host threads and their work (included in
+       the totals above) */
+    int64_t cpu_ends, cpu_inserts, cpu_walk_steps, cpu_attempts;
 } la_stats;
 
 la_status la_create(la_ctx **out, int device, void *cuda_stream /* cudaStream_t; NULL: own stream */);
@@ -175,6 +178,14 @@ la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const char *conti
  * of the last la_extend are unchanged.  Errors: LA_ERR_STATE if no la_extend completed since the
  * last la_load_batch; LA_ERR_CUDA (sticky). */
 la_status la_replay_build(la_ctx *ctx);
+/* CPU+GPU co-execution (the paper's co-scheduling of LA on CPU cores and
+ * GPUs, §4.3, Fig 11): with n_threads > 0 and cpu_share > 0, every following la_extend /
+ * la_extend_device / la_extend_streamed gives the lightest round(cpu_share x n) ends of the smallest
+ * table class (n ends; by the planner's work estimate) to n_threads host threads, which extend them
+ * (a host implementation of the same method, in this library) while the GPU's kernels run; the
+ * results are identical and are returned with the GPU's.  n_threads = 0 or cpu_share = 0 turns it
+ * off (the default).  Errors: LA_ERR_INVALID_ARG unless 0 <= n_threads <= 1024, 0 <= cpu_share <= 1. */
+la_status la_set_coexec(la_ctx *ctx, int32_t n_threads, double cpu_share);
 la_status la_get_stats(const la_ctx *ctx, la_stats *out);
 la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
 const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */

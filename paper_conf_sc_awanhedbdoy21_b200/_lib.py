@@ -55,11 +55,13 @@ class la_stats(ctypes.Structure):
                 ("ms_build", ctypes.c_double), ("ms_walk", ctypes.c_double),
                 ("cls_build_ms", ctypes.c_double * 6), ("cls_build_inserts", ctypes.c_int64 * 6),
                 ("cls_inl_attempts", ctypes.c_int64 * 6), ("cls_ref_attempts", ctypes.c_int64 * 6),
-                ("attempts_hist", ctypes.c_int64 * LA_HIST), ("cls_dead0", ctypes.c_int64 * 6)]
+                ("attempts_hist", ctypes.c_int64 * LA_HIST), ("cls_dead0", ctypes.c_int64 * 6),
+                ("cpu_ends", ctypes.c_int64), ("cpu_inserts", ctypes.c_int64), ("cpu_walk_steps", ctypes.c_int64),
+                ("cpu_attempts", ctypes.c_int64)]
 
 
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
-           "la_replay_build",
+           "la_replay_build", "la_set_coexec",
            "la_get_stats", "la_destroy", "la_last_error", "la_plan_global_capacity", "la_paper_load_factor"]
 
 _lib = None
@@ -90,6 +92,7 @@ def load():
     lib.la_append_extensions.argtypes = [V, ctypes.c_int32, V, V, V, V, V, V]
     lib.la_get_stats.argtypes = [V, ctypes.POINTER(la_stats)]
     lib.la_replay_build.argtypes = [V]
+    lib.la_set_coexec.argtypes = [V, ctypes.c_int32, ctypes.c_double]
     lib.la_destroy.argtypes = [V]
     lib.la_last_error.argtypes = [V]
     lib.la_last_error.restype = ctypes.c_char_p
@@ -98,7 +101,7 @@ def load():
     lib.la_paper_load_factor.argtypes = [ctypes.c_int32, ctypes.c_int32]
     lib.la_paper_load_factor.restype = ctypes.c_double
     for f in ("la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
-              "la_replay_build", "la_get_stats", "la_destroy"):
+              "la_replay_build", "la_set_coexec", "la_get_stats", "la_destroy"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib

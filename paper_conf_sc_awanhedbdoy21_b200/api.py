@@ -188,6 +188,12 @@ class LocalAssembler:
                                                    eoff_ptr, eseq_ptr, out_seq.data_ptr(), out_off.data_ptr()))
         return out_seq[:tot], out_off
 
+    def set_coexec(self, n_threads: int, cpu_share: float):
+        """la_set_coexec: NEXT N3 CPU+GPU co-execution (the lightest ends of the smallest class on host
+        threads while the GPU runs); n_threads = 0 turns it off."""
+        self._check(self._lib.la_set_coexec(self._ctx, int(n_threads), float(cpu_share)))
+        return self
+
     def replay_build(self) -> dict:
         """la_replay_build: rerun the last extension's table builds only (the hash-build phase) and
         return the stats with ms_build / cls_build_ms / cls_build_inserts filled in."""

@@ -12,8 +12,9 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SO = os.path.join(HERE, "liblocassm.so")
-SRC = [os.path.join(HERE, "csrc", "locassm.cu")]
-DEPS = SRC + sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu*"))) + [os.path.join(ROOT, "include", "locassm.h")]
+SRC = [os.path.join(HERE, "csrc", "locassm.cu"), os.path.join(HERE, "csrc", "la_cpu.cpp")]
+DEPS = SRC + sorted(glob.glob(os.path.join(HERE, "csrc", "*.cu*")) + glob.glob(os.path.join(HERE, "csrc", "*.h")) +
+                   glob.glob(os.path.join(HERE, "csrc", "*.cpp"))) + [os.path.join(ROOT, "include", "locassm.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-shared", "-Xcompiler", "-fPIC", "-I" + os.path.join(ROOT, "include")]

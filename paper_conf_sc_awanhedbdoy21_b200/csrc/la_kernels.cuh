@@ -202,6 +202,55 @@ namespace la {
 // ------------------------------------------------------------------------------------------------
 // emit (a9)
 // ------------------------------------------------------------------------------------------------
+// ---- NEXT N3 co-execution: gather the host's ends, scatter its results ----
+__global__ void k_cx_counts(const int32_t *__restrict__ list, int m, const int64_t *__restrict__ eoff,
+                            int64_t *__restrict__ cnt) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < m) cnt[i] = eoff[list[i] + 1] - eoff[list[i]];
+    else if (i == m) cnt[i] = 0;
+}
+// one warp per end: its reads' packed rows, lengths, and the contig tail
+__global__ void k_cx_gather(const int32_t *__restrict__ list, int m, const int64_t *__restrict__ eoff,
+                            const int64_t *__restrict__ goff, int SW, const uint64_t *__restrict__ rseq,
+                            const uint64_t *__restrict__ rqc, const uint16_t *__restrict__ rlen,
+                            const uint64_t *__restrict__ tail, const uint64_t *__restrict__ tailN,
+                            const int32_t *__restrict__ clen, uint64_t *__restrict__ g_rseq,
+                            uint64_t *__restrict__ g_rqc, uint16_t *__restrict__ g_rlen, uint64_t *__restrict__ g_tail,
+                            uint64_t *__restrict__ g_tailN, int32_t *__restrict__ g_clen) {
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int i = (int)(t >> 5), lane = (int)(t & 31);
+    if (i >= m) return;
+    const int e = list[i];
+    const int64_t r0 = eoff[e], n = eoff[e + 1] - r0, g0 = goff[i];
+    for (int64_t w = lane; w < n * SW; w += 32) {
+        g_rseq[g0 * SW + w] = rseq[r0 * SW + w];
+        g_rqc[g0 * SW + w] = rqc[r0 * SW + w];
+    }
+    for (int64_t j = lane; j < n; j += 32) g_rlen[g0 + j] = rlen[r0 + j];
+    if (lane < TAIL_W) g_tail[(int64_t)i * TAIL_W + lane] = tail[(int64_t)e * TAIL_W + lane];
+    if (lane < 2) g_tailN[2 * (int64_t)i + lane] = tailN[2 * (int64_t)e + lane];
+    if (lane == 0) g_clen[i] = clen[e];
+}
+__global__ void k_cx_scatter(const int32_t *__restrict__ list, int m, int W, const int32_t *__restrict__ len,
+                             const uint8_t *__restrict__ term, const uint8_t *__restrict__ kk,
+                             const uint8_t *__restrict__ att, const int8_t *__restrict__ dir,
+                             const uint8_t *__restrict__ walk, int32_t *__restrict__ out_len,
+                             uint8_t *__restrict__ out_term, uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att,
+                             int8_t *__restrict__ out_dir, uint8_t *__restrict__ walk_buf) {
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int i = (int)(t >> 5), lane = (int)(t & 31);
+    if (i >= m) return;
+    const int e = list[i];
+    for (int j = lane; j < len[i]; j += 32) walk_buf[(int64_t)e * W + j] = walk[(int64_t)i * W + j];
+    if (lane == 0) {
+        out_len[e] = len[i];
+        out_term[e] = term[i];
+        out_k[e] = kk[i];
+        out_att[e] = att[i];
+        out_dir[e] = dir[i];
+    }
+}
+
 // ends per attempt count (la_stats.attempts_hist; the last bin collects >= LA_HIST - 1)
 __global__ void k_att_hist(const uint8_t *__restrict__ att, int64_t n, unsigned long long *__restrict__ hist) {
     __shared__ unsigned int h[LA_HIST];

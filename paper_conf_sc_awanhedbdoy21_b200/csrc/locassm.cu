@@ -15,6 +15,7 @@
 #include <vector>
 
 #include "locassm.h"
+#include "la_cpu.h"
 #include "la_kernels.cuh"
 
 using namespace la;
@@ -108,6 +109,13 @@ struct la_ctx {
     DevBuf g_state, g_act, g_act2, g_still, g_cap, g_nrd, g_capoff, g_rdoff, g_slots, g_cnt, g_vis,
         g_cur;
     DevBuf lens64, xl_scratch, prof, out_dir, hist;
+    // NEXT N3 co-execution (la_set_coexec): host threads, share of the smallest class's ends, buffers
+    int coexec_threads = 0;
+    double coexec_share = 0.0;
+    DevBuf cx_cnt, cx_roff, cx_rseq, cx_rqc, cx_rlen, cx_tail, cx_tailN, cx_clen, cx_len, cx_term, cx_k, cx_att,
+        cx_dir, cx_walk;
+    HostBuf hx_roff, hx_rseq, hx_rqc, hx_rlen, hx_tail, hx_tailN, hx_clen, hx_len, hx_term, hx_k, hx_att, hx_dir,
+        hx_walk;
     // plan of the last la_extend (la_replay_build reruns its class lists)
     bool extended = false;
     int plan_ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
@@ -333,7 +341,14 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
                       &ctx->glob_list, &ctx->ctrs, &ctx->ext_off, &ctx->ext_seq, &ctx->gstats,
                       &ctx->cub_tmp, &ctx->g_state, &ctx->g_act, &ctx->g_act2, &ctx->g_still, &ctx->g_cap,
                       &ctx->g_nrd, &ctx->g_capoff, &ctx->g_rdoff, &ctx->g_slots, &ctx->g_cnt, &ctx->g_vis,
-                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch, &ctx->prof, &ctx->out_dir, &ctx->hist})
+                      &ctx->g_cur, &ctx->lens64, &ctx->xl_scratch, &ctx->prof, &ctx->out_dir, &ctx->hist,
+                      &ctx->cx_cnt, &ctx->cx_roff, &ctx->cx_rseq, &ctx->cx_rqc, &ctx->cx_rlen, &ctx->cx_tail,
+                      &ctx->cx_tailN, &ctx->cx_clen, &ctx->cx_len, &ctx->cx_term, &ctx->cx_k, &ctx->cx_att,
+                      &ctx->cx_dir, &ctx->cx_walk})
+        b->release();
+    for (HostBuf *b : {&ctx->hx_roff, &ctx->hx_rseq, &ctx->hx_rqc, &ctx->hx_rlen, &ctx->hx_tail, &ctx->hx_tailN,
+                       &ctx->hx_clen, &ctx->hx_len, &ctx->hx_term, &ctx->hx_k, &ctx->hx_att, &ctx->hx_dir,
+                       &ctx->hx_walk})
         b->release();
     for (HostBuf *b : {&ctx->h_ext_off, &ctx->h_ext_seq, &ctx->h_term, &ctx->h_k, &ctx->h_att, &ctx->h_small})
         b->release();
@@ -693,6 +708,111 @@ la_status launch_classes(la_ctx *ctx, bool replay) {
     return LA_OK;
 }
 
+// ---- NEXT N3: CPU+GPU co-execution (la_set_coexec) ---------------------------------------------
+// The lightest ends of the smallest table class (the tail of its LPT-sorted list) are gathered on the
+// device into compact arrays, copied to pinned host memory and extended by la_cpu::extend on host
+// threads while the GPU's class kernels run; their results are copied back and scattered into the
+// device result arrays, so the device compaction emits every end the same way.
+struct Coexec {
+    int m = 0;                 // ends given to the host
+    const int32_t *list = nullptr;   // their ids (device, the class list's tail)
+    int64_t reads = 0;
+};
+
+la_status coexec_gather(la_ctx *ctx, int32_t *d_list, int m, Coexec &cx) {
+    cudaStream_t st = ctx->stream;
+    Encoded &E = ctx->enc;
+    const int SW = E.SW;
+    cx.m = m;
+    cx.list = d_list;
+    CK(grow(ctx->cx_cnt, (size_t)(m + 1) * 8));
+    CK(grow(ctx->cx_roff, (size_t)(m + 1) * 8));
+    k_cx_counts<<<blocks(m + 1, 256), 256, 0, st>>>(d_list, m, P<int64_t>(E.eoff), P<int64_t>(ctx->cx_cnt));
+    CKL();
+    size_t tb = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, tb, P<int64_t>(ctx->cx_cnt), P<int64_t>(ctx->cx_roff), m + 1, st);
+    CK(grow(ctx->cub_tmp, tb));
+    cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, P<int64_t>(ctx->cx_cnt), P<int64_t>(ctx->cx_roff), m + 1, st);
+    CKL();
+    CK(grow_host(ctx->hx_roff, (size_t)(m + 1) * 8));
+    CK(cudaMemcpyAsync(ctx->hx_roff.p, ctx->cx_roff.p, (size_t)(m + 1) * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const int64_t R = ((int64_t *)ctx->hx_roff.p)[m];
+    cx.reads = R;
+    CK(grow(ctx->cx_rseq, (size_t)std::max<int64_t>(R, 1) * SW * 8));
+    CK(grow(ctx->cx_rqc, (size_t)std::max<int64_t>(R, 1) * SW * 8));
+    CK(grow(ctx->cx_rlen, (size_t)std::max<int64_t>(R, 1) * 2));
+    CK(grow(ctx->cx_tail, (size_t)m * TAIL_W * 8));
+    CK(grow(ctx->cx_tailN, (size_t)m * 16));
+    CK(grow(ctx->cx_clen, (size_t)m * 4));
+    k_cx_gather<<<blocks((int64_t)m * 32, 256), 256, 0, st>>>(
+        d_list, m, P<int64_t>(E.eoff), P<int64_t>(ctx->cx_roff), SW, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
+        P<uint16_t>(E.rlen), P<uint64_t>(E.tail), P<uint64_t>(E.tailN), P<int32_t>(E.clen), P<uint64_t>(ctx->cx_rseq),
+        P<uint64_t>(ctx->cx_rqc), P<uint16_t>(ctx->cx_rlen), P<uint64_t>(ctx->cx_tail), P<uint64_t>(ctx->cx_tailN),
+        P<int32_t>(ctx->cx_clen));
+    CKL();
+    CK(grow_host(ctx->hx_rseq, (size_t)std::max<int64_t>(R, 1) * SW * 8));
+    CK(grow_host(ctx->hx_rqc, (size_t)std::max<int64_t>(R, 1) * SW * 8));
+    CK(grow_host(ctx->hx_rlen, (size_t)std::max<int64_t>(R, 1) * 2));
+    CK(grow_host(ctx->hx_tail, (size_t)m * TAIL_W * 8));
+    CK(grow_host(ctx->hx_tailN, (size_t)m * 16));
+    CK(grow_host(ctx->hx_clen, (size_t)m * 4));
+    if (R) {
+        CK(cudaMemcpyAsync(ctx->hx_rseq.p, ctx->cx_rseq.p, (size_t)R * SW * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(ctx->hx_rqc.p, ctx->cx_rqc.p, (size_t)R * SW * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(ctx->hx_rlen.p, ctx->cx_rlen.p, (size_t)R * 2, cudaMemcpyDeviceToHost, st));
+    }
+    CK(cudaMemcpyAsync(ctx->hx_tail.p, ctx->cx_tail.p, (size_t)m * TAIL_W * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(ctx->hx_tailN.p, ctx->cx_tailN.p, (size_t)m * 16, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(ctx->hx_clen.p, ctx->cx_clen.p, (size_t)m * 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    return LA_OK;
+}
+
+// host extension of the gathered ends (runs while the class kernels execute), then results -> device
+la_status coexec_finish(la_ctx *ctx, const Coexec &cx) {
+    cudaStream_t st = ctx->stream;
+    const DevParams &dp = ctx->dp;
+    const int m = cx.m, W = std::max(dp.W, 1);
+    CK(grow_host(ctx->hx_len, (size_t)m * 4));
+    CK(grow_host(ctx->hx_term, (size_t)m));
+    CK(grow_host(ctx->hx_k, (size_t)m));
+    CK(grow_host(ctx->hx_att, (size_t)m));
+    CK(grow_host(ctx->hx_dir, (size_t)m));
+    CK(grow_host(ctx->hx_walk, (size_t)m * W));
+    la_cpu::Input in{m, ctx->enc.SW, (const int64_t *)ctx->hx_roff.p, (const uint64_t *)ctx->hx_rseq.p,
+                     (const uint64_t *)ctx->hx_rqc.p, (const uint16_t *)ctx->hx_rlen.p,
+                     (const uint64_t *)ctx->hx_tail.p, (const uint64_t *)ctx->hx_tailN.p,
+                     (const int32_t *)ctx->hx_clen.p};
+    la_cpu::Output out{(int32_t *)ctx->hx_len.p, (uint8_t *)ctx->hx_walk.p, (uint8_t *)ctx->hx_term.p,
+                       (uint8_t *)ctx->hx_k.p, (uint8_t *)ctx->hx_att.p, (int8_t *)ctx->hx_dir.p, 0, 0, 0};
+    la_cpu::Params cp{dp.k_start, dp.k_min, dp.k_max, dp.k_shift, dp.W, dp.V, dp.F};
+    la_cpu::extend(in, cp, ctx->coexec_threads, out);
+    ctx->stats.cpu_ends = m;
+    ctx->stats.cpu_inserts = out.inserts;
+    ctx->stats.cpu_walk_steps = out.walk_steps;
+    ctx->stats.cpu_attempts = out.attempts;
+    CK(grow(ctx->cx_len, (size_t)m * 4));
+    CK(grow(ctx->cx_term, (size_t)m));
+    CK(grow(ctx->cx_k, (size_t)m));
+    CK(grow(ctx->cx_att, (size_t)m));
+    CK(grow(ctx->cx_dir, (size_t)m));
+    CK(grow(ctx->cx_walk, (size_t)m * W));
+    CK(cudaMemcpyAsync(ctx->cx_len.p, ctx->hx_len.p, (size_t)m * 4, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(ctx->cx_term.p, ctx->hx_term.p, (size_t)m, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(ctx->cx_k.p, ctx->hx_k.p, (size_t)m, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(ctx->cx_att.p, ctx->hx_att.p, (size_t)m, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(ctx->cx_dir.p, ctx->hx_dir.p, (size_t)m, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(ctx->cx_walk.p, ctx->hx_walk.p, (size_t)m * W, cudaMemcpyHostToDevice, st));
+    k_cx_scatter<<<blocks((int64_t)m * 32, 256), 256, 0, st>>>(
+        cx.list, m, W, P<int32_t>(ctx->cx_len), P<uint8_t>(ctx->cx_term), P<uint8_t>(ctx->cx_k),
+        P<uint8_t>(ctx->cx_att), P<int8_t>(ctx->cx_dir), P<uint8_t>(ctx->cx_walk), P<int32_t>(ctx->out_len),
+        P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), P<int8_t>(ctx->out_dir),
+        P<uint8_t>(ctx->walk_buf));
+    CKL();
+    return LA_OK;
+}
+
 la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     if (!ctx || !out) return LA_ERR_INVALID_ARG;
     if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
@@ -781,6 +901,16 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         CKL();
         CK(cudaMemcpyAsync(lst, ctx->smem_list2.p, (size_t)n * 4, cudaMemcpyDeviceToDevice, st));
     }
+    // NEXT N3: the lightest ends of the smallest class (its list's tail) go to the host threads
+    Coexec cx;
+    if (ctx->coexec_threads > 0 && ctx->coexec_share > 0.0 && ncls[0] > 0) {
+        const int m = (int)std::min<double>(ncls[0], std::floor(ctx->coexec_share * ncls[0] + 0.5));
+        if (m > 0) {
+            ncls[0] -= m;
+            const la_status s0 = coexec_gather(ctx, lists + ncls[0], m, cx);
+            if (s0 != LA_OK) return s0;
+        }
+    }
     CK(cudaEventRecord(ctx->ev[1], st));
     ctx->plan_nxl = n_xl;
     ctx->plan_xl_umax = xl_umax;
@@ -789,6 +919,10 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
     {
         const la_status s0 = launch_classes(ctx, false);
+        if (s0 != LA_OK) return s0;
+    }
+    if (cx.m) {   // the host's share, while the class kernels run
+        const la_status s0 = coexec_finish(ctx, cx);
         if (s0 != LA_OK) return s0;
     }
     int n_ovf = 0;
@@ -847,10 +981,10 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     const int64_t total = h64[0];
     // d_gst: [0] smem inserts [1] smem walk steps [2] smem attempts [3] global inserts [4] global steps
-    ctx->stats.inserts = h64[1] + h64[4];
+    ctx->stats.inserts = h64[1] + h64[4] + ctx->stats.cpu_inserts;
     ctx->stats.inserts_smem = h64[1];
-    ctx->stats.walk_steps = h64[2] + h64[5];
-    ctx->stats.attempts = h64[3] + ctx->g_attempts;
+    ctx->stats.walk_steps = h64[2] + h64[5] + ctx->stats.cpu_walk_steps;
+    ctx->stats.attempts = h64[3] + ctx->g_attempts + ctx->stats.cpu_attempts;
     ctx->stats.ext_bases = total;
     CK(grow(ctx->ext_seq, total + 16));
     if (nE) {
@@ -901,7 +1035,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         ctx->stats.cls_ms[c] = m;
     }
     // class counts (host-side tally from the plan counters)
-    ctx->stats.ends_by_class[2] = n_smem - n_ovf;
+    ctx->stats.ends_by_class[2] = n_smem - n_ovf + cx.m;   // the host's ends are counted with class 0
     ctx->stats.ends_by_class[3] = n_glob;
     ctx->stats.ends_by_class[4] = n_ovf;
     ctx->stats.ends_medium = ncls[3] + ncls[4];
@@ -1086,6 +1220,10 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
             acc.ends_medium += x.ends_medium;
             acc.ms_smem_medium += x.ms_smem_medium;
             acc.ends_xl += x.ends_xl;
+            acc.cpu_ends += x.cpu_ends;
+            acc.cpu_inserts += x.cpu_inserts;
+            acc.cpu_walk_steps += x.cpu_walk_steps;
+            acc.cpu_attempts += x.cpu_attempts;
             acc.xl_scratch_bytes = std::max(acc.xl_scratch_bytes, x.xl_scratch_bytes);
             for (int q = 0; q < 6; ++q) {
                 acc.cls_ends[q] += x.cls_ends[q];
@@ -1120,6 +1258,15 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
     return LA_OK;
 }
 extern "C" la_status la_extend_device(la_ctx *ctx, la_result *out) { return extend_impl(ctx, out, false); }
+
+extern "C" la_status la_set_coexec(la_ctx *ctx, int32_t n_threads, double cpu_share) {
+    if (!ctx) return LA_ERR_INVALID_ARG;
+    if (n_threads < 0 || n_threads > 1024 || !(cpu_share >= 0.0 && cpu_share <= 1.0))
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_set_coexec: need 0 <= n_threads <= 1024 and 0 <= cpu_share <= 1");
+    ctx->coexec_threads = n_threads;
+    ctx->coexec_share = cpu_share;
+    return LA_OK;
+}
 
 // Build-only replay (SURVEY §8(d) timing protocol step 5): the table-class kernels rerun, over the
 // class lists of the last la_extend, exactly the (end, k) attempts it made (k_start + i * shift for

@@ -372,3 +372,30 @@ def test_xl_wide_counters(LA, orc):
         sub = C.Batch.from_lists([contig], ends)
         _, st = check(LA, orc, sub, P0, env={"LA_FORCE_CLASS": "5"})
         assert st["cls_inl_attempts"][5] > 0 and st["ends_by_class"][4] == 0
+
+
+@pytest.mark.parametrize("share", [1.0, 0.3])
+def test_coexec_matches_oracle(LA, orc, share):
+    """NEXT N3: the lightest ends of the smallest class extended on host threads while the GPU runs
+    (la_set_coexec) — every end still bit-exact against the oracle, work counters included."""
+    b = cached_batch("C2", scale=0.03)
+    LA.set_coexec(8, share)
+    try:
+        r, st = check(LA, orc, b, P0)
+    finally:
+        LA.set_coexec(0, 0.0)
+    assert st["cpu_ends"] > 0 and st["cpu_inserts"] > 0
+    r2 = LA.extend()   # co-execution off: same results, no host ends
+    assert r2.ext_list() == r.ext_list() and LA.stats()["cpu_ends"] == 0
+
+
+def test_coexec_streamed(LA, orc, c2_ref):
+    b, ref = c2_ref
+    LA.set_coexec(4, 0.5)
+    try:
+        r = LA.extend_streamed(b, P0, 3)
+        st = LA.stats()
+    finally:
+        LA.set_coexec(0, 0.0)
+    assert r.ext_list() == ref["ext"] and np.array_equal(r.term, ref["term"])
+    assert st["cpu_ends"] > 0 and st["inserts"] == int(ref["inserts"].sum())
