@@ -468,6 +468,50 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
     }
 }
 
+// Dynamic version for ends whose reads all have length ulen > 0: warps take chunks of 32 * UNR
+// consecutive positions from a shared counter (one atomic per chunk) instead of a fixed 1/nwarps
+// range, so no warp waits at the pass's closing barrier for a slower one (probe rounds differ).
+template <int NW, int UNR, typename F>
+__device__ __forceinline__ void warp_positions32_dyn(const uint32_t *__restrict__ rseq, const uint32_t *__restrict__ rqc,
+                                                     const uint8_t *__restrict__ rflag, uint32_t total, long long r0,
+                                                     int SW2, int k, int ulen, int lane, const volatile int *stop,
+                                                     int *ctr, F &&f) {
+    const KMask m = kmask32<NW>(k);
+    const uint32_t np = (uint32_t)(ulen - k);
+    const uint32_t magic = 0xFFFFFFFFu / np;
+    for (;;) {
+        uint32_t base = 0;
+        if (lane == 0) base = (uint32_t)atomicAdd(ctr, 32 * UNR);
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (base >= total || __shfl_sync(0xffffffffu, *stop, 0)) return;
+#pragma unroll
+        for (int u = 0; u < UNR; ++u) {
+            const uint32_t gu = base + 32u * u + lane;
+            const bool act = gu < total;
+            uint32_t jj = __umulhi(gu, magic);
+            uint32_t pp = gu - jj * np;
+            if (pp >= np) { ++jj; pp -= np; }
+            const int p = act ? (int)pp : 0;
+            const long long row = (r0 + (act ? (int)jj : 0)) * (long long)SW2;
+            const uint32_t *R = rseq + row, *Q = rqc + row;
+            const K32<NW> K = extract32<NW>(R, p, m);
+            const uint32_t nb = base32(R, p + k), nq = base32(Q, p + k);
+            bool vote = act && (nq - 1u < 2u);
+            if (vote && rflag[r0 + jj]) {   // reading #5: a k-mer with an N has no entry (rare)
+                const int q = p >> 4, s = (p & 15) << 1;
+                uint32_t any = 0;
+#pragma unroll
+                for (int w = 0; w < NW; ++w) {
+                    const uint32_t mw = w == NW - 1 ? m.m1 : (w == NW - 2 ? m.m2 : ~0u);
+                    any |= __funnelshift_l(nmask32(rw32(Q, q + w + 1)), nmask32(rw32(Q, q + w)), s) & mw;
+                }
+                if (any) vote = false;
+            }
+            f(act, vote, gu, K, hash32<NW>(K), nb, nq == 2u);
+        }
+    }
+}
+
 // (read, offset) of position g of the end (pref: positions per read, exclusive prefix)
 __device__ __forceinline__ void pos_of(uint32_t g, const uint32_t *pref, int r, int ulen, int k, int &j, int &p) {
     if (ulen > 0) {

@@ -48,6 +48,10 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_FILTER_UNROLL
 #define LA_FILTER_UNROLL 2   // positions per lane per iteration of the filter pass (la_inl32.cuh)
 #endif
+#ifndef LA_DYN
+#define LA_DYN 1   // dynamic 32-position chunks in the filter / build passes of the shared-memory classes
+                   // (warp_positions32_dyn; XL measured slower with them)
+#endif
 #ifndef LA_DEAD0
 #define LA_DEAD0 1   // decide attempts whose start k-mer fails the filter without building (inl32_build_link)
 #endif
@@ -600,6 +604,7 @@ struct BuildCtl {           // builders' shared scratch
     uint32_t start;
     uint32_t start_h;       // hash of the start k-mer (inline keys); start_ok: it has no N
     int start_ok, dead0;    // dead0: the attempt is decided before the build (start k-mer < 2 votes)
+    int ctr_f, ctr_b;       // position chunk counters of the filter / build pass (warp_positions32_dyn)
     int lmin, lmax;
     uint32_t wsum[32];      // per builder warp: prefix-scan totals
 };
@@ -732,8 +737,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     if (!mbits || !LA_FQUEUE) {
         if (mbits) {
             // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
-            warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
-                                 [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
+            auto filt = [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
                                      if (!act) return;
                                      const uint32_t fi = filt32(h, mbits);
                                      const uint32_t bit = 1u << (fi & 31);
@@ -747,7 +751,13 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                              if (old & bit) atomicOr(&B2[fi >> 5], bit);
                                          }
                                      }
-                                 });
+                                 };
+            if (LA_DYN && !GT && ulen > k)
+                warp_positions32_dyn<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref[r], r0, SW2, k, ulen, lane, stop,
+                                                           &B.ctr_f, filt);
+            else
+                warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
+                                                       stop, filt);
             builders_sync(NB);
             // The filter has no false negatives: a start k-mer whose B2 bit is clear has < 2 voting
             // occurrences, so with V >= 2 (filters are only used then) it extends to DEADEND at step 0
@@ -769,16 +779,18 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         t_filter = la_clock();
         // ---- build (Alg 1): every voting occurrence that passed the filter ----
         uint32_t pend = 0;   // carry check of this lane's last vote (vote32d)
-        warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop,
-                             [&](bool, bool act, uint32_t, const K32<NW> &K, uint32_t h, uint32_t nb, bool hi) {
-                                 bool want = act;
-                                 if (mbits) {
-                                     const uint32_t fi = filt32(h, mbits);
-                                     want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
-                                 }
-                                 warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim,
-                                                   claim_limit, &B.overflow, pend);
-                             });
+        auto build = [&](bool, bool act, uint32_t, const K32<NW> &K, uint32_t h, uint32_t nb, bool hi) {
+            bool want = act;
+            if (mbits) {
+                const uint32_t fi = filt32(h, mbits);
+                want = want && ((B2[fi >> 5] >> (fi & 31)) & 1u);
+            }
+            warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim, claim_limit, &B.overflow, pend);
+        };
+        if (LA_DYN && !GT && ulen > k)
+            warp_positions32_dyn<NW, 1>(R32, Q32, rflag, pref[r], r0, SW2, k, ulen, lane, stop, &B.ctr_b, build);
+        else
+            warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop, build);
         flush_vote32(pend, &B.overflow);
     } else {
         // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4); every position's
@@ -1133,6 +1145,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             B.overflow = 0;
             B.nclaim = 0;
             B.dead0 = 0;
+            B.ctr_f = B.ctr_b = 0;
             if (E.done) {   // refill the slot with the next end, or retire it
                 int idx, e = 0;
                 do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
@@ -1473,6 +1486,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 B.overflow = 0;
                 B.nclaim = 0;
                 B.dead0 = 0;
+                B.ctr_f = B.ctr_b = 0;
+            B.ctr_f = B.ctr_b = 0;
             }
             const long long tc = la_clock();
             {
