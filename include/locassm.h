@@ -52,6 +52,7 @@ typedef enum {
 typedef enum { LA_MEM_HOST = 0, LA_MEM_DEVICE = 1 } la_mem;
 
 #define LA_HIST 16
+#define LA_N_CLASSES 7
 
 typedef struct {
     int32_t k_start, k_min, k_max, k_shift; /* 1 <= k_min <= k_start <= k_max <= 128; k_shift >= 1 */
@@ -113,23 +114,26 @@ typedef struct {
     double ms_smem_medium;       /* summed kernel times of the XL, 2- and 1-CTA/SM classes          */
     int64_t ends_xl;             /* ends whose table lived in the XL class's global scratch        */
     int64_t xl_scratch_bytes;
-    /* per table class: 0..4 shared memory (64, 128, 256@3, 256@2, 512 threads), 5 = XL */
-    int64_t cls_ends[6], cls_inserts[6], cls_attempts[6], cls_filtered[6];
-    double cls_ms[6];            /* device time of each class kernel (serial by default; spans if
+    /* per table class (LA_N_CLASSES): 0..4 shared memory (64x12, 128x6, 256x3, 512x2, 1024x1 threads x
+       CTAs per SM), 5 = XL (table in L2-resident global scratch), 6 = XLC (table split over a 2-CTA
+       cluster's shared memory, reached through DSMEM) */
+    int64_t cls_ends[LA_N_CLASSES], cls_inserts[LA_N_CLASSES], cls_attempts[LA_N_CLASSES],
+        cls_filtered[LA_N_CLASSES];
+    double cls_ms[LA_N_CLASSES];            /* device time of each class kernel (serial by default; spans if
                                     LA_CONCURRENT_CLASSES=1 launches them together)                */
     /* LA_PROFILE=1 only: per class, summed clock64 cycles of the builders' leader (wait for the
        walker, prefix, clear, filter pass, build pass, link) and of the walker (wait, walk) */
-    uint64_t prof_cycles[6][8];
+    uint64_t prof_cycles[LA_N_CLASSES][8];
     /* hash-build / walk split (SURVEY.md §8(b), §8(d) timing step 5), set by la_replay_build
        (-1 until then): ms_build = device time of the build-only replay of the table-class kernels,
        ms_walk = ms_smem - ms_build (link pass, walk and hand-offs); per class likewise */
     double ms_build, ms_walk;
-    double cls_build_ms[6];
-    int64_t cls_build_inserts[6];
+    double cls_build_ms[LA_N_CLASSES];
+    int64_t cls_build_inserts[LA_N_CLASSES];
     /* per class: attempts built with inline keys (k <= 63) and with pointer keys (k >= 64) */
-    int64_t cls_inl_attempts[6], cls_ref_attempts[6];
+    int64_t cls_inl_attempts[LA_N_CLASSES], cls_ref_attempts[LA_N_CLASSES];
     int64_t attempts_hist[LA_HIST]; /* ends by number of attempts (last bin: >= LA_HIST-1)       */
-    int64_t cls_dead0[6];   /* per class: attempts decided after the filter pass (the start k-mer has
+    int64_t cls_dead0[LA_N_CLASSES];   /* per class: attempts decided after the filter pass (the start k-mer has
                                < 2 voting occurrences: DEADEND at step 0 without building the table) */
     /* NEXT N3 co-execution (la_set_coexec): ends extended on host threads and their work (included in
        the totals above) */

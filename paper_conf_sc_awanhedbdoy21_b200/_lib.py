@@ -14,6 +14,7 @@ SO = os.environ.get("LA_SO") or os.path.join(HERE, "liblocassm.so")   # LA_SO: d
 LA_OK, LA_ERR_INVALID_ARG, LA_ERR_OOM, LA_ERR_CUDA, LA_ERR_STATE, LA_ERR_CAPACITY = 0, -1, -2, -3, -4, -5
 LA_MEM_HOST, LA_MEM_DEVICE = 0, 1
 LA_HIST = 16
+LA_N_CLASSES = 7   # 0-4 shared memory, 5 XL, 6 XLC
 STATUS = {0: "LA_OK", -1: "LA_ERR_INVALID_ARG", -2: "LA_ERR_OOM", -3: "LA_ERR_CUDA",
           -4: "LA_ERR_STATE", -5: "LA_ERR_CAPACITY"}
 TERM_NAMES = ["DEADEND", "FORK", "LOOP", "MAXLEN", "NOREADS", "SHORT"]
@@ -48,14 +49,14 @@ class la_stats(ctypes.Structure):
                 ("smem_bytes_per_cta", ctypes.c_int64), ("smem_ctas_per_sm", ctypes.c_int32),
                 ("global_rounds", ctypes.c_int32), ("ends_medium", ctypes.c_int64),
                 ("ms_smem_medium", ctypes.c_double), ("ends_xl", ctypes.c_int64),
-                ("xl_scratch_bytes", ctypes.c_int64), ("cls_ends", ctypes.c_int64 * 6),
-                ("cls_inserts", ctypes.c_int64 * 6), ("cls_attempts", ctypes.c_int64 * 6),
-                ("cls_filtered", ctypes.c_int64 * 6), ("cls_ms", ctypes.c_double * 6),
-                ("prof_cycles", (ctypes.c_uint64 * 8) * 6),
+                ("xl_scratch_bytes", ctypes.c_int64), ("cls_ends", ctypes.c_int64 * LA_N_CLASSES),
+                ("cls_inserts", ctypes.c_int64 * LA_N_CLASSES), ("cls_attempts", ctypes.c_int64 * LA_N_CLASSES),
+                ("cls_filtered", ctypes.c_int64 * LA_N_CLASSES), ("cls_ms", ctypes.c_double * LA_N_CLASSES),
+                ("prof_cycles", (ctypes.c_uint64 * 8) * LA_N_CLASSES),
                 ("ms_build", ctypes.c_double), ("ms_walk", ctypes.c_double),
-                ("cls_build_ms", ctypes.c_double * 6), ("cls_build_inserts", ctypes.c_int64 * 6),
-                ("cls_inl_attempts", ctypes.c_int64 * 6), ("cls_ref_attempts", ctypes.c_int64 * 6),
-                ("attempts_hist", ctypes.c_int64 * LA_HIST), ("cls_dead0", ctypes.c_int64 * 6),
+                ("cls_build_ms", ctypes.c_double * LA_N_CLASSES), ("cls_build_inserts", ctypes.c_int64 * LA_N_CLASSES),
+                ("cls_inl_attempts", ctypes.c_int64 * LA_N_CLASSES), ("cls_ref_attempts", ctypes.c_int64 * LA_N_CLASSES),
+                ("attempts_hist", ctypes.c_int64 * LA_HIST), ("cls_dead0", ctypes.c_int64 * LA_N_CLASSES),
                 ("cpu_ends", ctypes.c_int64), ("cpu_inserts", ctypes.c_int64), ("cpu_walk_steps", ctypes.c_int64),
                 ("cpu_attempts", ctypes.c_int64)]
 

@@ -195,6 +195,7 @@ __global__ void k_encode_tails(const char *__restrict__ cseq, const int64_t *__r
 }  // namespace la
 
 #include "la_smem.cuh"
+#include "la_xlc.cuh"
 #include "la_global.cuh"
 
 namespace la {

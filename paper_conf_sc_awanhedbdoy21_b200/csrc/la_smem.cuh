@@ -193,6 +193,56 @@ __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_
     return T;
 }
 
+// ---- XLC class (la_xlc.cuh): one end per 2-CTA cluster, table split over both SMs (DSMEM) ----
+constexpr int XLC_THREADS = 1024;
+constexpr uint32_t XLC_MAX_U = 65535u;   // 16-bit counter fields cannot carry below this
+// Shared-memory layout of each CTA: [stage reads (if staged)][pref][B1 half | B2 half][keys half]
+// [counters half][claim list][rank 0: info (cap x u32)] ... [2 walk strings at the end of the region,
+// fixed across attempts].  Identical in both CTAs (info unused in rank 1), from (r, U, bytes, stage).
+struct XlcLayout {
+    uint32_t off_pref, off_b1, off_b2, off_keys, off_cnts, off_list, off_info, off_walk;
+    uint32_t cap, half, hw, mwords;
+    bool fits;
+};
+__host__ __device__ __forceinline__ float xlc_filtered_fraction(int r) {
+    return r < 50 ? 0.30f : (r < 200 ? 0.16f : 0.10f);   // as the planner's filtered_fraction
+}
+__host__ __device__ __forceinline__ XlcLayout xlc_layout(uint32_t bytes, int r, int SW, uint32_t U, int W, bool stage) {
+    XlcLayout L;
+    const uint32_t Wp = ((uint32_t)(W > 0 ? W : 1) + 15u) & ~15u;
+    const uint32_t sb = ((uint32_t)r * (uint32_t)SW * 16u + (uint32_t)r * 3u + 15u) & ~15u;
+    const uint32_t pb = (((uint32_t)r + 1u) * 4u + 15u) & ~15u;
+    const float est = (float)U * xlc_filtered_fraction(r) + 1024.f;   // filtered keys + margin, load <= 0.7
+    // (no in-flight margin: warp_insert_c bounds every probe sequence, a full table overflows)
+    uint32_t cap = ((uint32_t)(est / SMEM_MAX_LOAD) + 3u) & ~3u;
+    if (cap < 4096u) cap = 4096u;
+    L.cap = cap;
+    L.half = cap / 2u;
+    L.mwords = ((4u * U + 31u) / 32u + 7u) & ~7u;   // words of each bitmap (4 bits per occurrence)
+    L.hw = L.mwords / 2u;
+    L.off_walk = bytes > 2u * Wp ? ((bytes - 2u * Wp) & ~15u) : 0u;
+    uint32_t o = stage ? sb : 0u;
+    L.off_pref = o;
+    o += pb;
+    L.off_b1 = o;
+    o += L.hw * 4u;
+    L.off_b2 = o;
+    o += L.hw * 4u;
+    o = (o + 15u) & ~15u;
+    L.off_keys = o;
+    o += L.half * 16u;
+    L.off_cnts = o;
+    o += L.half * 16u;
+    L.off_list = o;
+    o += cap * 2u;   // one CTA may claim up to its limit (0.45 cap) of the whole table
+    o = (o + 15u) & ~15u;
+    L.off_info = o;
+    o += cap * 4u;
+    L.fits = o <= L.off_walk && U <= XLC_MAX_U && L.half <= 32768u && bytes > 2u * Wp;
+    return L;
+}
+
+
 // ---- plan ------------------------------------------------------------------------------------
 // Routing estimate of the filtered table: distinct k-mers with >= 2 voting occurrences plus filter
 // false positives, as a fraction of the occurrences (measured on C2/C4 samples: 0.05-0.2, higher for
@@ -220,6 +270,8 @@ __device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, u
 // (512, 2), (1024, 1); one warp of each CTA walks, the others build.  The first class whose table is
 // predicted to fit wins; G = global-memory rounds.
 constexpr int N_SMEM_CLASSES = 5;
+constexpr int C_XLC = N_SMEM_CLASSES + 1;   // class indices: 0-4 shared memory, 5 XL, 6 XLC
+constexpr int N_TAB_CLASSES = N_SMEM_CLASSES + 2;
 struct PlanBytes {
     uint32_t b[N_SMEM_CLASSES];   // dynamic shared memory per CTA
     uint32_t t[N_SMEM_CLASSES];   // threads per CTA
@@ -249,11 +301,12 @@ __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_
 
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
                        const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW, PlanBytes pb,
-                       uint32_t xl_bytes, int force_cls,
+                       uint32_t xl_bytes, uint32_t xlc_bytes, int force_cls,
                        int32_t *__restrict__ cls, int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
                        uint8_t *__restrict__ out_k, uint8_t *__restrict__ out_att, int32_t *__restrict__ lists,
                        uint32_t *__restrict__ keys, int32_t *__restrict__ list_G, int *__restrict__ ctr) {
-    // ctr: [0..4] n per smem class, [5] n_G, [6] NOREADS, [7] SHORT, [8] n_XL, [9] max U_XL, [10] max r_XL
+    // ctr: [0..4] n per smem class, [5] n_G, [6] NOREADS, [7] SHORT, [8] n_XL, [9] max U_XL, [10] max r_XL,
+    // [11] n_XLC
     const int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (e >= n_ends) return;
     const int64_t r = eoff[e + 1] - eoff[e];
@@ -275,6 +328,10 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
             for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
                 if (fits(r, U, P, pb.b[i], pb.t[i], SW, (pb.single >> i) & 1u)) sc = i;
         U0 = U0 > 0xffffffffll ? 0xffffffffll : U0;
+        // XLC: the table split over a 2-CTA cluster's shared memory (no staging assumed; U < 65536)
+        if (sc < 0 && xlc_bytes && P.V >= 2 && r <= 16384 && U <= XLC_MAX_U &&
+            xlc_layout(xlc_bytes, (int)r, SW, (uint32_t)U, P.W, false).fits)
+            sc = C_XLC;
         if (sc < 0 && xl_bytes && r <= 16384 && U <= XL_MAX_U &&
             xl_needed_cap(r, U, P.V >= 2) <= smem_fixed(P.W, xl_bytes, 1u, false, XL_THREADS / 32 - 1).icap)
             sc = N_SMEM_CLASSES;   // XL: table in global scratch
@@ -283,7 +340,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         if (force_cls >= 0 && r <= 16384 && U <= XL_MAX_U) sc = force_cls;
         if (sc >= 0) {
             c = CLS_S + sc;
-            const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : sc], 1);
+            const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : (sc == C_XLC ? 11 : sc)], 1);
             lists[sc * n_ends + i] = (int32_t)e;
             keys[sc * n_ends + i] = (uint32_t)U0;
             if (sc == N_SMEM_CLASSES) {

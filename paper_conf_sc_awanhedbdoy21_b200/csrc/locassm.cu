@@ -119,7 +119,9 @@ struct la_ctx {
     // plan of the last la_extend (la_replay_build reruns its class lists)
     bool extended = false;
     int plan_ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
-    int plan_nxl = 0, plan_xl_umax = 0, plan_xl_rmax = 0;
+    int plan_nxl = 0, plan_xl_umax = 0, plan_xl_rmax = 0, plan_nxlc = 0;
+    uint32_t xlc_bytes = 0;   // dynamic shared memory per CTA of the XLC cluster class (0: not planned)
+    uint32_t xlc_force_bytes = 0;   // the same for LA_FORCE_CLASS=6
     HostBuf h_ext_off, h_ext_seq, h_term, h_k, h_att, h_small;
     // la_extend_streamed: copy stream, double-buffered raw staging (A/B), chunk-ordering events
     cudaStream_t copy_stream = nullptr;
@@ -128,11 +130,11 @@ struct la_ctx {
     int64_t g_attempts = 0;
     cudaEvent_t ev[6] = {};
     cudaEvent_t ev_rep[2] = {};   // la_replay_build start / end
-    cudaEvent_t ev_cls[N_SMEM_CLASSES + 2] = {};   // end of class c; [N] end of XL; [N+1] classes may start
-    cudaEvent_t ev_cls0[N_SMEM_CLASSES + 1] = {};  // start of class c ([N] = XL)
+    cudaEvent_t ev_cls[N_TAB_CLASSES + 1] = {};   // end of class c (5 XL, 6 XLC); [N_TAB_CLASSES] classes may start
+    cudaEvent_t ev_cls0[N_TAB_CLASSES] = {};      // start of class c
     // one stream per table class (LA_CONCURRENT_CLASSES=1): the persistent class kernels launched together (largest tables
     // first) so that the tail of one class overlaps the start of the next; LA_SERIAL_CLASSES=1: one stream
-    cudaStream_t cls_stream[N_SMEM_CLASSES + 1] = {};
+    cudaStream_t cls_stream[N_TAB_CLASSES] = {};
     // r02: the class kernels run one after another on the context stream by default.  Measured on C4S,
     // launching them on six streams at once gave the same step time (each persistent class kernel
     // fills the GPU, so only their tails can overlap) while making the per-class times overlapping
@@ -312,6 +314,13 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
         for (const ClassEntry &k : kClassKernels)
             attr_ok &= cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) == cudaSuccess;
     }
+    // XLC (2-CTA clusters, la_xlc.cuh): opt-in (LA_XLC=1).  Measured on C4S it ran its ends at 21 G
+    // inserts/s against the XL class's 36 (step 140.2 vs 130.6 ms), so the planner does not route ends to
+    // it by default; LA_FORCE_CLASS=6 (tests) forces it.
+    ctx->xlc_bytes = (getenv("LA_XLC") && atoi(getenv("LA_XLC"))) ? ctx->cls_bytes[N_SMEM_CLASSES - 1] : 0u;
+    ctx->xlc_force_bytes = ctx->cls_bytes[N_SMEM_CLASSES - 1];
+    attr_ok &= cudaFuncSetAttribute(k_xlc, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->cls_bytes[N_SMEM_CLASSES - 1]) ==
+               cudaSuccess;
     if (!attr_ok) {
         cudaGetLastError();
         la_destroy(ctx);
@@ -649,16 +658,29 @@ la_status launch_classes(la_ctx *ctx, bool replay) {
     // LA_PROFILE=1: per-class phase cycle counters (clock64) of the shared-memory kernels
     unsigned long long *prof = nullptr;
     if (!replay && getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE"))) {
-        CK(grow(ctx->prof, 8 * 8 * (N_SMEM_CLASSES + 1)));
+        CK(grow(ctx->prof, 8 * 8 * N_TAB_CLASSES));
         prof = P<unsigned long long>(ctx->prof);
-        CK(cudaMemsetAsync(prof, 0, 8 * 8 * (N_SMEM_CLASSES + 1), st));
+        CK(cudaMemsetAsync(prof, 0, 8 * 8 * N_TAB_CLASSES, st));
     }
-    CK(cudaEventRecord(ctx->ev_cls[N_SMEM_CLASSES + 1], st));
+    CK(cudaEventRecord(ctx->ev_cls[N_TAB_CLASSES], st));
     auto cls_st = [&](int c) -> cudaStream_t {
         return (ctx->concurrent_classes && ctx->cls_stream[c]) ? ctx->cls_stream[c] : st;
     };
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c)
-        if (cls_st(c) != st) CK(cudaStreamWaitEvent(cls_st(c), ctx->ev_cls[N_SMEM_CLASSES + 1], 0));
+    for (int c = 0; c < N_TAB_CLASSES; ++c)
+        if (cls_st(c) != st) CK(cudaStreamWaitEvent(cls_st(c), ctx->ev_cls[N_TAB_CLASSES], 0));
+    // XLC (2-CTA clusters, tables in the pair's shared memory) first
+    CK(cudaEventRecord(ctx->ev_cls0[C_XLC], cls_st(C_XLC)));
+    if (ctx->plan_nxlc > 0) {
+        const int clusters = (int)std::min<int64_t>((int64_t)ctx->n_sm / 2, ctx->plan_nxlc);
+        k_xlc<<<2 * clusters, XLC_THREADS, ctx->xlc_force_bytes, cls_st(C_XLC)>>>(
+            lists + (size_t)C_XLC * nE, ctx->plan_nxlc, d_ctr + 22, P<uint64_t>(E.rseq), P<uint64_t>(E.rqc),
+            P<uint16_t>(E.rlen), P<uint8_t>(E.rflag), P<int64_t>(E.eoff), P<uint64_t>(E.tail), P<uint64_t>(E.tailN),
+            P<int32_t>(E.clen), E.SW, dp, ctx->xlc_force_bytes, P<uint8_t>(ctx->walk_buf), P<int32_t>(ctx->out_len),
+            P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att), P<int8_t>(ctx->out_dir),
+            ovf_list, d_ctr + 15, (GlobalStats *)(d_gst + 8 + GSTATS_WORDS * C_XLC));
+        CKL();
+    }
+    CK(cudaEventRecord(ctx->ev_cls[C_XLC], cls_st(C_XLC)));
     // XL (global-scratch tables) first, then the shared-memory classes from the largest tables
     // (1 CTA/SM, all shared memory) to the smallest (12 CTAs/SM)
     CK(cudaEventRecord(ctx->ev_cls0[N_SMEM_CLASSES], cls_st(N_SMEM_CLASSES)));
@@ -703,7 +725,7 @@ la_status launch_classes(la_ctx *ctx, bool replay) {
         }
         CK(cudaEventRecord(ctx->ev_cls[c], cls_st(c)));   // end of class c
     }
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c)   // join
+    for (int c = 0; c < N_TAB_CLASSES; ++c)   // join
         if (cls_st(c) != st) CK(cudaStreamWaitEvent(st, ctx->ev_cls[c], 0));
     return LA_OK;
 }
@@ -834,8 +856,8 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(grow(ctx->out_k, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->out_att, std::max<int64_t>(nE, 1)));
     CK(grow(ctx->walk_buf, std::max<int64_t>(nE, 1) * W));
-    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4 * (N_SMEM_CLASSES + 1)));
-    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4 * (N_SMEM_CLASSES + 1)));
+    CK(grow(ctx->smem_list, std::max<int64_t>(nE, 1) * 4 * N_TAB_CLASSES));
+    CK(grow(ctx->smem_key, std::max<int64_t>(nE, 1) * 4 * N_TAB_CLASSES));
     CK(grow(ctx->smem_list2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->smem_key2, std::max<int64_t>(nE, 1) * 4));
     CK(grow(ctx->glob_list, std::max<int64_t>(nE, 1) * 4 * 2));
@@ -853,7 +875,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     CK(cudaMemsetAsync(d_gst, 0, 512, st));
     int *h = (int *)ctx->h_small.p;
     int ncls[N_SMEM_CLASSES] = {0, 0, 0, 0, 0};
-    int n_glob = 0, n_xl = 0, xl_umax = 0, xl_rmax = 0;
+    int n_glob = 0, n_xl = 0, xl_umax = 0, xl_rmax = 0, n_xlc = 0;
     int32_t *lists = P<int32_t>(ctx->smem_list);
     uint32_t *keys = P<uint32_t>(ctx->smem_key);
     if (nE) {
@@ -869,14 +891,16 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         pb.single = ctx->small_mask;
         if (force_smem) pb.b[0] = 0xffffffffu;
         // test hook: every end with reads into table class LA_FORCE_CLASS (0..4 shared memory, 5 = XL)
-        const int force_cls = getenv("LA_FORCE_CLASS") ? std::min(std::max(atoi(getenv("LA_FORCE_CLASS")), 0), 5) : -1;
+        const int force_cls = getenv("LA_FORCE_CLASS") ? std::min(std::max(atoi(getenv("LA_FORCE_CLASS")), 0), 6) : -1;
+        const uint32_t xlc_b = force_cls == C_XLC ? ctx->xlc_force_bytes : ctx->xlc_bytes;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
             P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
-            (force_global || force_smem) ? 0u : ctx->xl_bytes, force_global ? -1 : force_cls, P<int32_t>(ctx->cls),
+            (force_global || force_smem) ? 0u : ctx->xl_bytes, (force_global || force_smem) ? 0u : xlc_b,
+            force_global ? -1 : force_cls, P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
             lists, keys, P<int32_t>(ctx->glob_list), d_ctr);
         CKL();
-        CK(cudaMemcpyAsync(h, d_ctr, 4 * 11, cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(h, d_ctr, 4 * 12, cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
         for (int i = 0; i < N_SMEM_CLASSES; ++i) ncls[i] = h[i];
         n_glob = h[N_SMEM_CLASSES];
@@ -885,10 +909,11 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         n_xl = h[8];
         xl_umax = h[9];
         xl_rmax = h[10];
+        n_xlc = h[11];
     }
     // LPT order for the persistent kernels: largest expected work first
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
-        const int n = c == N_SMEM_CLASSES ? n_xl : ncls[c];
+    for (int c = 0; c < N_TAB_CLASSES; ++c) {
+        const int n = c == N_SMEM_CLASSES ? n_xl : (c == C_XLC ? n_xlc : ncls[c]);
         if (n < 2) continue;
         int32_t *lst = lists + (size_t)c * nE;
         uint32_t *key = keys + (size_t)c * nE;
@@ -915,6 +940,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     ctx->plan_nxl = n_xl;
     ctx->plan_xl_umax = xl_umax;
     ctx->plan_xl_rmax = xl_rmax;
+    ctx->plan_nxlc = n_xlc;
     for (int c = 0; c < N_SMEM_CLASSES; ++c) ctx->plan_ncls[c] = ncls[c];
     int32_t *ovf_list = P<int32_t>(ctx->glob_list) + nE;
     {
@@ -926,7 +952,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         if (s0 != LA_OK) return s0;
     }
     int n_ovf = 0;
-    int n_smem = n_xl;
+    int n_smem = n_xl + n_xlc;
     for (int c = 0; c < N_SMEM_CLASSES; ++c) n_smem += ncls[c];
     if (n_smem > 0) {
         CK(cudaMemcpyAsync(h, d_ctr + 15, 4, cudaMemcpyDeviceToHost, st));
@@ -958,7 +984,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     int64_t *h64 = (int64_t *)ctx->h_small.p;
     CK(cudaMemcpyAsync(h64, P<int64_t>(ctx->ext_off) + nE, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(h64 + 1, d_gst, 8 * (8 + GSTATS_WORDS * (N_SMEM_CLASSES + 1)), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64 + 1, d_gst, 8 * (8 + GSTATS_WORDS * N_TAB_CLASSES), cudaMemcpyDeviceToHost, st));
     CK(cudaMemcpyAsync(h64 + 64, ctx->hist.p, 8 * LA_HIST, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (getenv("LA_PROFILE") && atoi(getenv("LA_PROFILE")) && ctx->prof.p) {
@@ -966,9 +992,9 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     }
     // per-class stats (classes 0..4 shared memory, 5 = XL); fold them into the smem totals
     for (int i = 0; i < LA_HIST; ++i) ctx->stats.attempts_hist[i] = h64[64 + i];
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
+    for (int c = 0; c < N_TAB_CLASSES; ++c) {
         const int64_t *g = h64 + 1 + 8 + GSTATS_WORDS * c;
-        ctx->stats.cls_ends[c] = c < N_SMEM_CLASSES ? ncls[c] : n_xl;
+        ctx->stats.cls_ends[c] = c < N_SMEM_CLASSES ? ncls[c] : (c == C_XLC ? n_xlc : n_xl);
         ctx->stats.cls_inserts[c] = g[0];
         ctx->stats.cls_attempts[c] = g[2];
         ctx->stats.cls_filtered[c] = g[3];
@@ -1029,7 +1055,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
     ctx->stats.ms_global = ms;
     cudaEventElapsedTime(&ms, ctx->ev[3], ctx->ev[4]);
     ctx->stats.ms_emit = ms;
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {   // start -> end of each class kernel (they may overlap)
+    for (int c = 0; c < N_TAB_CLASSES; ++c) {   // start -> end of each class kernel
         float m = 0;
         cudaEventElapsedTime(&m, ctx->ev_cls0[c], ctx->ev_cls[c]);
         ctx->stats.cls_ms[c] = m;
@@ -1225,7 +1251,7 @@ extern "C" la_status la_extend_streamed(la_ctx *ctx, const la_batch *b, const la
             acc.cpu_walk_steps += x.cpu_walk_steps;
             acc.cpu_attempts += x.cpu_attempts;
             acc.xl_scratch_bytes = std::max(acc.xl_scratch_bytes, x.xl_scratch_bytes);
-            for (int q = 0; q < 6; ++q) {
+            for (int q = 0; q < N_TAB_CLASSES; ++q) {
                 acc.cls_ends[q] += x.cls_ends[q];
                 acc.cls_inserts[q] += x.cls_inserts[q];
                 acc.cls_attempts[q] += x.cls_attempts[q];
@@ -1280,20 +1306,20 @@ extern "C" la_status la_replay_build(la_ctx *ctx) {
     cudaStream_t st = ctx->stream;
     int *d_ctr = P<int>(ctx->ctrs);
     unsigned long long *d_gst = P<unsigned long long>(ctx->gstats);
-    CK(cudaMemsetAsync(d_ctr + 15, 0, 4 * 8, st));   // overflow count + the class work counters
-    CK(cudaMemsetAsync(d_gst + 8, 0, 8 * GSTATS_WORDS * (N_SMEM_CLASSES + 1), st));
+    CK(cudaMemsetAsync(d_ctr + 15, 0, 4 * 8, st));   // overflow count + the class work counters (16..22)
+    CK(cudaMemsetAsync(d_gst + 8, 0, 8 * GSTATS_WORDS * N_TAB_CLASSES, st));
     CK(cudaEventRecord(ctx->ev_rep[0], st));
     const la_status s = launch_classes(ctx, true);
     if (s != LA_OK) return s;
     CK(cudaEventRecord(ctx->ev_rep[1], st));
     int64_t *h64 = (int64_t *)ctx->h_small.p;
-    CK(cudaMemcpyAsync(h64, d_gst + 8, 8 * GSTATS_WORDS * (N_SMEM_CLASSES + 1), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h64, d_gst + 8, 8 * GSTATS_WORDS * N_TAB_CLASSES, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     float ms = 0;
     cudaEventElapsedTime(&ms, ctx->ev_rep[0], ctx->ev_rep[1]);
     ctx->stats.ms_build = ms;
     ctx->stats.ms_walk = ctx->stats.ms_smem - ms;   // the rest of the table phase: link + walk + hand-offs
-    for (int c = 0; c <= N_SMEM_CLASSES; ++c) {
+    for (int c = 0; c < N_TAB_CLASSES; ++c) {
         float m = 0;
         cudaEventElapsedTime(&m, ctx->ev_cls0[c], ctx->ev_cls[c]);
         ctx->stats.cls_build_ms[c] = m;

@@ -313,14 +313,29 @@ def test_append_extensions_alignments(LA, seed):
     assert _appended_strings(seq, off) == oracle.append_extensions(contigs, ext)
 
 
-@pytest.mark.parametrize("cls", range(6))
+@pytest.mark.parametrize("cls", range(7))
 def test_class_by_key_format_matrix(LA, orc, cls):
-    """Every table class (0-4 shared memory, 5 = XL in global scratch) with inline keys (k <= 63) and
-    pointer keys (k >= 64), each forced (LA_FORCE_CLASS) and compared with the oracle end by end."""
+    """Every table class (0-4 shared memory, 5 = XL in global scratch, 6 = XLC split over a 2-CTA
+    cluster) with inline keys (k <= 63) and pointer keys (k >= 64), each forced (LA_FORCE_CLASS) and
+    compared with the oracle end by end.  XLC builds inline keys only: its ends with a k >= 64 attempt
+    are redone by the global rounds (still bit-exact)."""
     b = cached_batch("C2", scale=0.03).select_contigs(np.arange(400))
     for P, key in ((P0, "cls_inl_attempts"), (Params(k_start=65, k_min=57, k_max=97), "cls_ref_attempts")):
         _, st = check(LA, orc, b, P, env={"LA_FORCE_CLASS": str(cls)})
-        assert st[key][cls] > 0, (cls, key, st[key])
+        if cls == 6 and key == "cls_ref_attempts":   # k 65 first: every end goes on to the global rounds
+            assert st["ends_by_class"][4] > 0
+        else:
+            assert st[key][cls] > 0, (cls, key, st[key])
+
+
+def test_xlc_cluster_class(LA, orc):
+    """XLC (2-CTA cluster, table in both SMs' shared memory): C3's densest non-hot ends and the C2 slice
+    forced into it, bit-exact; and the planner routes ends there on its own."""
+    b = cached_batch("C2", scale=0.03)
+    _, st = check(LA, orc, b, P0, env={"LA_FORCE_CLASS": "6"})
+    assert st["cls_ends"][6] > 0 and st["cls_inl_attempts"][6] > 0
+    _, st = check(LA, orc, b, P0)
+    assert st["cls_ends"][6] == 0   # opt-in (LA_XLC=1): not planned by default (DESIGN.md §7)
 
 
 def test_replay_build_reruns_the_attempts(LA, orc):

@@ -20,7 +20,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--ends", type=int, default=2000)
-    ap.add_argument("--classes", default="none,0,1,2,3,4,5")
+    ap.add_argument("--classes", default="none,0,1,2,3,4,5,6")
     a = ap.parse_args()
     import oracle
     from gen import Params, make
