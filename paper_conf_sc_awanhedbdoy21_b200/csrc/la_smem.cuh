@@ -662,6 +662,7 @@ struct BuildCtl {           // builders' shared scratch
     uint32_t start_h;       // hash of the start k-mer (inline keys); start_ok: it has no N
     int start_ok, dead0;    // dead0: the attempt is decided before the build (start k-mer < 2 votes)
     int ctr_f, ctr_b;       // position chunk counters of the filter / build pass (warp_positions32_dyn)
+    SmemTab tb;             // this attempt's table layout, computed once by the leader (integer divisions)
     int lmin, lmax;
     uint32_t wsum[32];      // per builder warp: prefix-scan totals
 };
@@ -1052,7 +1053,12 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
     __shared__ __align__(8) uint64_t built[2], walked[2];   // mbarriers: slot s built / walked
     __shared__ unsigned long long s_acc[GSTATS_WORDS];   // work counters (GlobalStats order)
     const int tid = threadIdx.x;
-    const SmemFixed FX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u, false, NB / 32);
+    // the fixed layout lives in shared memory: computed once, read with LDS (kept in registers, the
+    // 64-register classes rematerialised its divisions inside the loops: ~4% of their instructions)
+    __shared__ SmemFixed sFX;
+    if (threadIdx.x == 0) sFX = smem_fixed(P.W, smem_bytes, GT ? gstride : 0u, false, NB / 32);
+    __syncthreads();
+    const SmemFixed &FX = sFX;
     // table region: shared memory, or this CTA's slice of the global scratch (XL class)
     unsigned char *tbase = GT ? gscratch + (size_t)blockIdx.x * gstride : sm;
     const int Wp = (P.W + 15) & ~15;
@@ -1323,16 +1329,21 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 FXt.filt_bytes -= xs;
             }
         }
-        SmemTab TB = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW);
-        if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
-            const uint32_t need = max(xl_needed_cap(r, U, TB.mwords != 0), min_table_cap(BLOCK));
-            if (TB.cap > need) {
-                TB.cap = (need + 1u) & ~1u;
-                TB.off_cnts = TB.off_keys + TB.cap * key_bytes(k);   // counters follow the keys
-                TB.off_list = TB.off_cnts + TB.cap * cnt_bytes(true, xl_wide(U));
-                TB.off_f = (TB.off_list + TB.cap * 2u + 15u) & ~15u;
+        if (bt == 0) {   // the attempt's table layout, once (broadcast through shared memory)
+            SmemTab tb = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW);
+            if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
+                const uint32_t need = max(xl_needed_cap(r, U, tb.mwords != 0), min_table_cap(BLOCK));
+                if (tb.cap > need) {
+                    tb.cap = (need + 1u) & ~1u;
+                    tb.off_cnts = tb.off_keys + tb.cap * key_bytes(k);   // counters follow the keys
+                    tb.off_list = tb.off_cnts + tb.cap * cnt_bytes(true, xl_wide(U));
+                    tb.off_f = (tb.off_list + tb.cap * 2u + 15u) & ~15u;
+                }
             }
+            B.tb = tb;
         }
+        builders_sync(NB);
+        const SmemTab TB = B.tb;
         bool ovf = no_room || TB.cap < min_table_cap(BLOCK);   // no room at this k (claims + in-flight < cap)
         if (!ovf) {
             const uint32_t mbits = TB.mwords * 32u;
@@ -1443,7 +1454,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
     __shared__ int s_done;
     __shared__ unsigned long long s_acc[GSTATS_WORDS];   // work counters (GlobalStats order)
     const int bt = threadIdx.x;
-    const SmemFixed FX = smem_fixed(P.W, smem_bytes, 0u, true, NB / 32);
+    __shared__ SmemFixed sFX;   // as in k_smem: computed once, read from shared memory
+    if (threadIdx.x == 0) sFX = smem_fixed(P.W, smem_bytes, 0u, true, NB / 32);
+    __syncthreads();
+    const SmemFixed &FX = sFX;
     const int Wp = (P.W + 15) & ~15;
     uint8_t *wstr = sm + FX.off_walk;   // two walk strings: current / best
     uint32_t *info = (uint32_t *)sm;
@@ -1516,7 +1530,9 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             const int KW = kwords(k);
             read_prefix(B, E, pref, sL, 0, r, k, E.ulen, bt, NB);
             const uint32_t U = pref[r];
-            SmemTab TB = smem_tab(FX, U, P.V >= 2, key_bytes(k), r, false, SW);
+            if (bt == 0) B.tb = smem_tab(FX, U, P.V >= 2, key_bytes(k), r, false, SW);   // once per attempt
+            __syncthreads();
+            const SmemTab TB = B.tb;
             if (TB.cap < min_table_cap(BLOCK)) {
                 ovf = true;
                 break;
