@@ -272,10 +272,21 @@ extern "C" la_status la_create(la_ctx **out, int device, void *cuda_stream) {
             fprintf(stderr, "locassm: LA_CLASSES / LA_SMALL_MASK names a class without a kernel; using defaults\n");
         }
     }
-    // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each)
+    // dynamic smem per CTA: the SM's shared memory split between resident CTAs (1 KB reserved each),
+    // minus the largest static shared memory of the class kernels (queried, not assumed)
+    size_t stat = 512;
+    {
+        cudaFuncAttributes fa;
+        for (const ClassEntry &k : kClassKernels)
+            if (cudaFuncGetAttributes(&fa, k.fn) == cudaSuccess) stat = std::max(stat, fa.sharedSizeBytes);
+        if (cudaFuncGetAttributes(&fa, k_smem<XL_THREADS, true>) == cudaSuccess) stat = std::max(stat, fa.sharedSizeBytes);
+        if (cudaFuncGetAttributes(&fa, k_xlc) == cudaSuccess) stat = std::max(stat, fa.sharedSizeBytes);
+        cudaGetLastError();
+        stat = (stat + 127) & ~(size_t)127;
+    }
     for (int i = 0; i < N_SMEM_CLASSES; ++i) {
-        size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - 512 /* static */;
-        per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - 512);
+        size_t per = prop.sharedMemPerMultiprocessor / ctx->cls_ctas[i] - 1024 - stat;
+        per = std::min(per, (size_t)prop.sharedMemPerBlockOptin - stat);
         ctx->cls_bytes[i] = (uint32_t)(per & ~(size_t)127);
     }
     // XL: tables live in L2; shared memory holds the link words and filter bitmaps, and whatever the
