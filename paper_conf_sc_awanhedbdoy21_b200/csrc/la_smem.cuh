@@ -747,6 +747,38 @@ __device__ __forceinline__ void read_prefix(BuildCtl &B, EndSlot &E, uint32_t *p
     }
 }
 
+// The walk (Alg 2) over the link words of one attempt, by one thread: loop check before
+// the lookup (reading #12, the visited bit), fork / dead end from the decided code (reading #1), at
+// most W bases (reading #7).  Bases are packed four to a 32-bit store (wb 4-byte aligned).  Returns the
+// walk length; term and the lookups made (a lookup per step, the LOOP step excluded) by reference.
+__device__ __forceinline__ int walk_links(uint32_t *info, uint32_t node, int W, uint8_t *wb, int &term,
+                                          unsigned long long &steps) {
+    int i = 0;
+    uint32_t pack = 0;
+    term = T_MAXLEN;
+    for (; i < W; ++i) {
+        if (node == NEXT_NONE) {
+            term = T_DEADEND;
+            break;
+        }
+        const uint32_t inf = info[node], code = inf & 7u;
+        if ((inf & 8u) | (code >= 4u)) {   // visited (loop check before the lookup) / fork / dead end
+            term = (inf & 8u) ? T_LOOP : (code == CODE_FORK ? T_FORK : T_DEADEND);
+            break;
+        }
+        info[node] = inf | 8u;
+        pack |= ((0x54474341u >> (8 * code)) & 0xffu) << (8 * (i & 3));   // "ACGT"[code]
+        if ((i & 3) == 3) {
+            *(uint32_t *)(wb + i - 3) = pack;
+            pack = 0;
+        }
+        node = inf >> 4;
+    }
+    for (int j = i & ~3; j < i; ++j) wb[j] = (uint8_t)(pack >> (8 * (j & 3)));
+    steps = (term == T_LOOP || term == T_MAXLEN) ? (unsigned long long)i : (unsigned long long)i + 1ull;
+    return i;
+}
+
 // Slot-parallel pass after the build: ext(lo, hi) (reading #1, a5) and, for a base, the successor
 // k-mer's slot (next_kmer, Alg 2 line 15) -> info[s] = next << 4 | code.
 __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
@@ -1117,21 +1149,9 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 // ---- walk (Alg 2) over the successor links ----
                 uint32_t *info = (uint32_t *)(sm + (s ? FX.off_info1 : 0u));
                 uint8_t *wb = wstr + (2 * s + (E.best_buf ^ 1)) * Wp;
-                uint32_t node = E.start == NONE ? NEXT_NONE : E.start;
-                int len = 0, term = T_MAXLEN;
-                unsigned long long steps = 0;
-                for (int i = 0; i < P.W; ++i) {
-                    ++steps;   // a lookup; the loop check of a present k-mer precedes it (below)
-                    if (node == NEXT_NONE) { term = T_DEADEND; break; }
-                    const uint32_t inf = info[node];
-                    if (inf & 8u) { term = T_LOOP; --steps; break; }   // visited: loop check before lookup
-                    info[node] = inf | 8u;
-                    const uint32_t code = inf & 7u;
-                    if (code == CODE_FORK) { term = T_FORK; break; }
-                    if (code == CODE_DEADEND) { term = T_DEADEND; break; }
-                    wb[len++] = (uint8_t)(0x54474341u >> (8 * code));   // "ACGT"[code] without a memory lookup
-                    node = inf >> 4;
-                }
+                int term;
+                unsigned long long steps;
+                const int len = walk_links(info, E.start == NONE ? NEXT_NONE : E.start, P.W, wb, term, steps);
                 E.attempts += 1;
                 E.steps += steps;
                 if (len > E.best_len) {   // longest walk, earliest on ties (reading #11)
@@ -1603,6 +1623,8 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 // ---- walk (Alg 2) over the successor links ----
                 E.ins += U;
                 uint8_t *wb = wstr + (E.best_buf ^ 1) * Wp;
+                // (k_small keeps the plain per-step loop: walk_links measured 5% slower here, where the
+                // walk's latency is exposed to the waiting CTA rather than its issue slots)
                 uint32_t node = B.start == NONE ? NEXT_NONE : B.start;
                 int len = 0, term = T_MAXLEN;
                 unsigned long long steps = 0;

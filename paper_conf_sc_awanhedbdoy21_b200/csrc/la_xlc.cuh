@@ -486,24 +486,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(XLC_THREADS, 1) k_xl
                     E.k += E.shift;
                 } else {
                     // ---- walk (Alg 2) over the link words, as k_small ----
-                    const uint32_t *info = (const uint32_t *)(sm + L.off_info);
-                    uint32_t *infow = (uint32_t *)(sm + L.off_info);
+                    uint32_t *info = (uint32_t *)(sm + L.off_info);
                     uint8_t *wb = wstr + (E.best_buf ^ 1) * Wp;
-                    uint32_t node = B.start == NONE ? NEXT_NONE : B.start;
-                    int len = 0, term = T_MAXLEN;
-                    unsigned long long steps = 0;
-                    for (int i = 0; i < P.W; ++i) {
-                        ++steps;
-                        if (node == NEXT_NONE) { term = T_DEADEND; break; }
-                        const uint32_t inf = info[node];
-                        if (inf & 8u) { term = T_LOOP; --steps; break; }
-                        infow[node] = inf | 8u;
-                        const uint32_t code = inf & 7u;
-                        if (code == CODE_FORK) { term = T_FORK; break; }
-                        if (code == CODE_DEADEND) { term = T_DEADEND; break; }
-                        wb[len++] = (uint8_t)(0x54474341u >> (8 * code));
-                        node = inf >> 4;
-                    }
+                    int term;
+                    unsigned long long steps;
+                    const int len = walk_links(info, B.start == NONE ? NEXT_NONE : B.start, P.W, wb, term, steps);
                     E.attempts += 1;
                     E.steps += steps;
                     if (len > E.best_len) {   // longest walk, earliest on ties (reading #11)
