@@ -207,7 +207,7 @@ namespace la {
 __global__ void k_cx_counts(const int32_t *__restrict__ list, int m, const int64_t *__restrict__ eoff,
                             int64_t *__restrict__ cnt) {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < m) cnt[i] = eoff[list[i] + 1] - eoff[list[i]];
+    if (i < m) cnt[i] = eoff[list_end(list[i]) + 1] - eoff[list_end(list[i])];
     else if (i == m) cnt[i] = 0;
 }
 // one warp per end: its reads' packed rows, lengths, and the contig tail
@@ -221,7 +221,7 @@ __global__ void k_cx_gather(const int32_t *__restrict__ list, int m, const int64
     const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int i = (int)(t >> 5), lane = (int)(t & 31);
     if (i >= m) return;
-    const int e = list[i];
+    const int e = list_end(list[i]);
     const int64_t r0 = eoff[e], n = eoff[e + 1] - r0, g0 = goff[i];
     for (int64_t w = lane; w < n * SW; w += 32) {
         g_rseq[g0 * SW + w] = rseq[r0 * SW + w];
@@ -241,7 +241,7 @@ __global__ void k_cx_scatter(const int32_t *__restrict__ list, int m, int W, con
     const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int i = (int)(t >> 5), lane = (int)(t & 31);
     if (i >= m) return;
-    const int e = list[i];
+    const int e = list_end(list[i]);
     for (int j = lane; j < len[i]; j += 32) walk_buf[(int64_t)e * W + j] = walk[(int64_t)i * W + j];
     if (lane == 0) {
         out_len[e] = len[i];

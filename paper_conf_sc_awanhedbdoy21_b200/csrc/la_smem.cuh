@@ -52,6 +52,9 @@ __device__ __forceinline__ long long la_clock() {
 #define LA_DYN 1   // dynamic 32-position chunks in the filter / build passes of the shared-memory classes
                    // (warp_positions32_dyn; XL measured slower with them)
 #endif
+#ifndef LA_ANYN
+#define LA_ANYN 1   // skip the per-position N test for ends without an N read (class list flag)
+#endif
 #ifndef LA_DEAD0
 #define LA_DEAD0 1   // decide attempts whose start k-mer fails the filter without building (inl32_build_link)
 #endif
@@ -299,7 +302,13 @@ __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_
             255u) & ~255u;
 }
 
+// class-list entries: the end id, bit 30 set when a read of the end has an N (list_end / list_anyn)
+constexpr int32_t LIST_ANYN = 1 << 30;
+__host__ __device__ __forceinline__ int list_end(int32_t v) { return v & (LIST_ANYN - 1); }
+__host__ __device__ __forceinline__ bool list_anyn(int32_t v) { return (v & LIST_ANYN) != 0; }
+
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
+                       const uint8_t *__restrict__ rflag,
                        const int32_t *__restrict__ clen, int64_t n_ends, DevParams P, int SW, PlanBytes pb,
                        uint32_t xl_bytes, uint32_t xlc_bytes, int force_cls,
                        int32_t *__restrict__ cls, int32_t *__restrict__ out_len, uint8_t *__restrict__ out_term,
@@ -317,10 +326,12 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         // exact voting-occurrence bounds U(k) = sum over reads of max(0, len - k) at the smallest k of
         // the schedule (table sizing) and at k_start (LPT key); reads shorter than k contribute 0
         int64_t U = 0, U0 = 0;
+        int anyN = 0;   // some read of the end has an N: only then do the passes test k-mer windows for N
         for (int64_t j = eoff[e]; j < eoff[e + 1]; ++j) {
             const int64_t l = roff[j + 1] - roff[j];
             U += l > P.k_min ? l - P.k_min : 0;
             U0 += l > P.k_start ? l - P.k_start : 0;
+            anyN |= rflag[j];
         }
         c = CLS_GLOBAL;
         int sc = -1;
@@ -341,7 +352,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         if (sc >= 0) {
             c = CLS_S + sc;
             const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : (sc == C_XLC ? 11 : sc)], 1);
-            lists[sc * n_ends + i] = (int32_t)e;
+            lists[sc * n_ends + i] = (int32_t)e | (anyN ? LIST_ANYN : 0);
             keys[sc * n_ends + i] = (uint32_t)U0;
             if (sc == N_SMEM_CLASSES) {
                 atomicMax(&ctr[9], (int)U);
@@ -652,6 +663,7 @@ struct EndSlot {            // one contig end in flight
     int done, dead, ovf;    // done: finished (refill); dead: no more ends; ovf: redo in the global path
     uint32_t start;         // the start k-mer's slot (NONE if absent) of the last build
     int rec_att;            // replay: attempts recorded by the extension
+    int anyN;               // some read of the end has an N (from the class list entry)
     unsigned long long ins, steps;
 };
 
@@ -793,7 +805,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                                  const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
                                                  int r, int ulen, const DevParams &P, const uint64_t *tail_e, int Tn,
                                                  uint64_t n0, uint64_t n1, int bt, int NB, long long &t_filter,
-                                                 long long &t_build, bool replay, void *fpos, uint32_t *queue) {
+                                                 long long &t_build, bool replay, void *fpos, uint32_t *queue, bool anyN) {
     const volatile int *stop = &B.overflow;
     const int k = TC.k;
     const int lane = bt & 31, wid = bt >> 5, nwarps = NB >> 5;
@@ -843,10 +855,10 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                      }
                                  };
             if (LA_DYN && !GT && ulen > k)
-                warp_positions32_dyn<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref[r], r0, SW2, k, ulen, lane, stop,
+                warp_positions32_dyn<NW, LA_FILTER_UNROLL>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
                                                            &B.ctr_f, filt);
             else
-                warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
+                warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
                                                        stop, filt);
             builders_sync(NB);
             // The filter has no false negatives: a start k-mer whose B2 bit is clear has < 2 voting
@@ -878,9 +890,9 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
             warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim, claim_limit, &B.overflow, pend);
         };
         if (LA_DYN && !GT && ulen > k)
-            warp_positions32_dyn<NW, 1>(R32, Q32, rflag, pref[r], r0, SW2, k, ulen, lane, stop, &B.ctr_b, build);
+            warp_positions32_dyn<NW, 1>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop, &B.ctr_b, build);
         else
-            warp_positions32<NW>(R32, Q32, rflag, pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop, build);
+            warp_positions32<NW>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop, build);
         flush_vote32(pend, &B.overflow);
     } else {
         // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4); every position's
@@ -979,18 +991,18 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                            const uint32_t *pref, long long r0, int r, const DevParams &P,
                                            const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, int bt, int NB,
                                            long long &t_filter, long long &t_build, bool replay, int ulen, void *fpos,
-                                           uint32_t *queue) {
+                                           uint32_t *queue, bool anyN) {
     if (INL) {
         const int nw = kw32(T.k);
         if (nw <= 2)
             inl32_build_link<2, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else if (nw == 3)
             inl32_build_link<3, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else
             inl32_build_link<4, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         return;
     }
     // ---- pointer keys (k >= 64): the same passes with 4-word k-mers ----
@@ -1230,16 +1242,20 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             B.dead0 = 0;
             B.ctr_f = B.ctr_b = 0;
             if (E.done) {   // refill the slot with the next end, or retire it
-                int idx, e = 0;
+                int idx, e = 0, lv = 0;
                 do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
                     idx = atomicAdd(work_ctr, 1);
-                    if (idx < n_list) e = list[idx];
+                    if (idx < n_list) {
+                        lv = list[idx];
+                        e = list_end(lv);
+                    }
                 } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
                 if (idx >= n_list) {
                     E.dead = 1;
                     mbar_arrive(&built[s]);   // the walker sees `dead` and retires the slot too
                 } else {
                     E.e = e;
+                    E.anyN = list_anyn(lv);
                     E.r0 = eoff[e];
                     E.r = (int)(eoff[e + 1] - E.r0);
                     E.ulen = -1;   // unknown until the first prefix pass
@@ -1405,10 +1421,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (INL)
                 build_link<true, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
+                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
             else
                 build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
+                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
             if (bt == 0) s_acc[6] += B.dead0;
         }
@@ -1486,14 +1502,18 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
     for (;;) {
         const long long ta = la_clock();
         if (bt == 0) {
-            int idx, e = 0;
+            int idx, e = 0, lv = 0;
             do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
                 idx = atomicAdd(work_ctr, 1);
-                if (idx < n_list) e = list[idx];
+                if (idx < n_list) {
+                        lv = list[idx];
+                        e = list_end(lv);
+                    }
             } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
             B.skip = idx >= n_list;
             if (!B.skip) {
                 E.e = e;
+                    E.anyN = list_anyn(lv);
                 E.r0 = eoff[e];
                 E.r = (int)(eoff[e + 1] - E.r0);
                 E.ulen = -1;
@@ -1598,10 +1618,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (inline_keys(k))
                 build_link<true, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                        NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
+                                        NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
             else
                 build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue);
+                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
             __syncthreads();
             const long long te = la_clock();
             b_t[1] += tc - tb;

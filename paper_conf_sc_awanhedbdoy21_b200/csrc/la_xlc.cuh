@@ -228,7 +228,7 @@ __device__ __forceinline__ void xlc_passes(BuildCtl &B, const TabC &T, uint32_t 
                                            long long lr0, int r, int SW, int k, int ulen, const DevParams &P,
                                            const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, uint32_t rank,
                                            int tid, int gw, int NWT, uint32_t flag_local, uint32_t flag_peer,
-                                           int claim_limit, bool replay) {
+                                           int claim_limit, bool replay, bool anyN) {
     const int lane = tid & 31;
     const uint32_t *R32 = (const uint32_t *)R64, *Q32 = (const uint32_t *)Q64;
     const int SW2 = 2 * SW;
@@ -251,7 +251,7 @@ __device__ __forceinline__ void xlc_passes(BuildCtl &B, const TabC &T, uint32_t 
     }
     // ---- filter pass (reading #4): B1 = seen once, B2 = seen at least twice, bitmaps split ----
     if (mbits) {
-        warp_positions32<NW, 2>(R32, Q32, gF, pref, lr0, r, SW2, k, ulen, gw, NWT, lane, stop,
+        warp_positions32<NW, 2>(R32, Q32, anyN ? gF : nullptr, pref, lr0, r, SW2, k, ulen, gw, NWT, lane, stop,
                                 [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
                                     if (!act) return;
                                     const uint32_t fi = filt32(h, mbits), bit = 1u << (fi & 31);
@@ -275,7 +275,7 @@ __device__ __forceinline__ void xlc_passes(BuildCtl &B, const TabC &T, uint32_t 
     __syncthreads();
     if (!B.dead0) {
         // ---- build (Alg 1) into the cluster table ----
-        warp_positions32<NW>(R32, Q32, gF, pref, lr0, r, SW2, k, ulen, gw, NWT, lane, stop,
+        warp_positions32<NW>(R32, Q32, anyN ? gF : nullptr, pref, lr0, r, SW2, k, ulen, gw, NWT, lane, stop,
                              [&](bool, bool act, uint32_t, const K32<NW> &K, uint32_t h, uint32_t nb, bool hi) {
                                  bool want = act;
                                  if (mbits) {
@@ -347,14 +347,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(XLC_THREADS, 1) k_xl
         // ---- rank 0 fetches the next end and pushes its slot to rank 1 ----
         if (tid == 0) s_umax = 0;
         if (rank == 0 && tid == 0) {
-            int idx, e = 0;
+            int idx, e = 0, lv = 0;
             do {   // replay: ends that left this kernel (overflow) in the extension are not replayed
                 idx = atomicAdd(work_ctr, 1);
-                if (idx < n_list) e = list[idx];
+                if (idx < n_list) {
+                        lv = list[idx];
+                        e = list_end(lv);
+                    }
             } while (P.replay && idx < n_list && out_dir[e] == OVF_DIR);
             E.dead = idx >= n_list;
             if (!E.dead) {
                 E.e = e;
+                E.anyN = list_anyn(lv);
                 E.r0 = eoff[e];
                 E.r = (int)(eoff[e + 1] - E.r0);
                 E.ulen = -1;
@@ -463,13 +467,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(XLC_THREADS, 1) k_xl
             const uint32_t mbits = L.mwords * 32u;
             if (NW <= 2)
                 xlc_passes<2>(B, T, mbits, gR, gQ, gF, pref, lr0, r, SW, k, E.ulen, P, tail_e, Tn, n0, n1, rank, tid,
-                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0);
+                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0, E.anyN != 0);
             else if (NW == 3)
                 xlc_passes<3>(B, T, mbits, gR, gQ, gF, pref, lr0, r, SW, k, E.ulen, P, tail_e, Tn, n0, n1, rank, tid,
-                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0);
+                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0, E.anyN != 0);
             else
                 xlc_passes<4>(B, T, mbits, gR, gQ, gF, pref, lr0, r, SW, k, E.ulen, P, tail_e, Tn, n0, n1, rank, tid,
-                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0);
+                              gw, NWT, flag_local, flag_peer, lim, P.replay != 0, E.anyN != 0);
             if (B.overflow) {   // identical in both CTAs (flags exchanged)
                 ovf = true;
                 break;

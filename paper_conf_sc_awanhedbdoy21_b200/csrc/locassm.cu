@@ -905,7 +905,7 @@ la_status extend_impl(la_ctx *ctx, la_result *out, bool to_host) {
         const int force_cls = getenv("LA_FORCE_CLASS") ? std::min(std::max(atoi(getenv("LA_FORCE_CLASS")), 0), 6) : -1;
         const uint32_t xlc_b = force_cls == C_XLC ? ctx->xlc_force_bytes : ctx->xlc_bytes;
         k_plan<<<blocks(nE, 256), 256, 0, st>>>(
-            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<int32_t>(E.clen), nE, dp, E.SW, pb,
+            P<int64_t>(E.eoff), P<int64_t>(E.roff), P<uint8_t>(E.rflag), P<int32_t>(E.clen), nE, dp, E.SW, pb,
             (force_global || force_smem) ? 0u : ctx->xl_bytes, (force_global || force_smem) ? 0u : xlc_b,
             force_global ? -1 : force_cls, P<int32_t>(ctx->cls),
             P<int32_t>(ctx->out_len), P<uint8_t>(ctx->out_term), P<uint8_t>(ctx->out_k), P<uint8_t>(ctx->out_att),
