@@ -29,10 +29,10 @@ class OrcParams(ctypes.Structure):
 
 def build(force: bool = False) -> str:
     """Compile oracle.cpp into liblaoracle.so (g++ -O2, single thread)."""
-    src = os.path.join(_HERE, "oracle.cpp")
+    srcs = [os.path.join(_HERE, "oracle.cpp"), os.path.join(_HERE, "select.cpp")]
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(
-            os.path.getmtime(src), os.path.getmtime(os.path.join(_HERE, "oracle.h"))):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", _SO, src])
+            [os.path.getmtime(p) for p in srcs] + [os.path.getmtime(os.path.join(_HERE, "oracle.h"))]):
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-o", _SO, *srcs])
     return _SO
 
 
@@ -47,6 +47,9 @@ def _load():
         lib.orc_extend.restype = ctypes.c_int
         lib.orc_ext_rule.argtypes = [P, P, P]
         lib.orc_ext_rule.restype = ctypes.c_int
+        lib.orc_select.argtypes = [ctypes.c_int32, P, P, ctypes.c_int64, P, P] + [ctypes.c_int32] * 5 + [
+            ctypes.c_int64, P, P, P]
+        lib.orc_select.restype = ctypes.c_int64
         _lib = lib
     return _lib
 
@@ -111,3 +114,56 @@ def append_extensions(contigs, ext):
     for c, seq in enumerate(contigs):
         out.append(ext[2 * c] + seq + ext[2 * c + 1])
     return out
+
+
+_COMP = bytes.maketrans(b"ACGTN", b"TGCAN")
+
+
+def select_reads(contig_seq, contig_off, read_seq, read_qual, read_off, w=150, s=16, t=4, o=20, mm_pct=4):
+    """NEXT N4, candidate-read selection (select.cpp, readings S1-S6 of DESIGN.md §10d): from a pool of
+    FR read pairs (reads 2i, 2i+1), the candidate reads of every contig end, written as la_load_batch
+    takes them.  Returns dict(end_read_off, read_seq, read_qual, read_off, sel_end, sel_pair, sel_flip).
+    S5-S6 (the batch layout) are written out here: per selected (end, pair) record in (end, pair)
+    order, mate 0 then mate 1, each reverse-complemented (qualities reversed) when its strand is -."""
+    lib = _load()
+    contig_seq = np.ascontiguousarray(contig_seq, np.uint8)
+    contig_off = np.ascontiguousarray(contig_off, np.int64)
+    read_seq = np.ascontiguousarray(read_seq, np.uint8)
+    read_qual = np.ascontiguousarray(read_qual, np.uint8)
+    read_off = np.ascontiguousarray(read_off, np.int64)
+    n_contigs = contig_off.shape[0] - 1
+    n_pairs = (read_off.shape[0] - 1) // 2
+    cap = max(16, 4 * n_pairs + 16)
+    while True:
+        se = np.zeros(cap, np.int64)
+        sp = np.zeros(cap, np.int64)
+        sf = np.zeros(cap, np.uint8)
+        n = lib.orc_select(n_contigs, _ptr(contig_seq), _ptr(contig_off), n_pairs, _ptr(read_seq), _ptr(read_off),
+                           int(w), int(s), int(t), int(o), int(mm_pct), cap, _ptr(se), _ptr(sp), _ptr(sf))
+        if n == -2:
+            cap *= 4
+            continue
+        if n < 0:
+            raise ValueError("oracle.select_reads: invalid arguments")
+        break
+    se, sp, sf = se[:n], sp[:n], sf[:n]
+    seq_out, qual_out, lens = [], [], []
+    rs, rq = read_seq.tobytes(), read_qual.tobytes()
+    for e, p, f in zip(se.tolist(), sp.tolist(), sf.tolist()):
+        for mate in (0, 1):
+            rid = 2 * p + mate
+            x, q = rs[read_off[rid]:read_off[rid + 1]], rq[read_off[rid]:read_off[rid + 1]]
+            flip = (mate == 0) == bool(f)     # f = 0: mate 0 as is, mate 1 rc'd; f = 1: the opposite
+            if flip:
+                x, q = x[::-1].translate(_COMP), q[::-1]
+            seq_out.append(x)
+            qual_out.append(q)
+            lens.append(len(x))
+    end_read_off = np.zeros(2 * n_contigs + 1, np.int64)
+    if n:
+        end_read_off[1:] = np.cumsum(2 * np.bincount(se, minlength=2 * n_contigs))
+    off = np.zeros(len(lens) + 1, np.int64)
+    off[1:] = np.cumsum(lens)
+    return dict(end_read_off=end_read_off, read_seq=np.frombuffer(b"".join(seq_out), np.uint8).copy(),
+                read_qual=np.frombuffer(b"".join(qual_out), np.uint8).copy(), read_off=off,
+                sel_end=se, sel_pair=sp, sel_flip=sf)
