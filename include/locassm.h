@@ -190,6 +190,55 @@ la_status la_replay_build(la_ctx *ctx);
  * results are identical and are returned with the GPU's.  n_threads = 0 or cpu_share = 0 turns it
  * off (the default).  Errors: LA_ERR_INVALID_ARG unless 0 <= n_threads <= 1024, 0 <= cpu_share <= 1. */
 la_status la_set_coexec(la_ctx *ctx, int32_t n_threads, double cpu_share);
+
+/* ---- NEXT N4: candidate-read selection ----
+ * The step before local assembly: "contigs are aligned against reads to find reads that can be used
+ * to further extend the contigs. The reads that align to the ends of contigs are then used for
+ * extending the contigs" (§2.2), left and right sides separately.  The paper
+ * gives no alignment rule; DESIGN.md §10d's readings S1-S6 define it:
+ *   S1 end window: the last `window` bases of the contig (RIGHT end 2c+1) / the first (LEFT end 2c);
+ *   S2 read x aligns to end e on strand σ (y = x or rc(x)) at diagonal d (y[j] faces C[d+j]) iff
+ *      (a) a stride seed y[j, j+seed_len), j = 0, seed_stride, 2*seed_stride, ..., lies inside the
+ *      window and equals the contig there (no N), (b) |[d, d+|y|) ∩ window| >= min_overlap,
+ *      (c) 100 x mismatches <= max_mism_pct x L over the whole contig overlap of length L (N mismatches);
+ *   S3 outward: RIGHT end: σ = + or the read reaches past the contig end; LEFT end: σ = - or it
+ *      starts before the contig start;
+ *   S4 pair i (reads 2i, 2i+1; an FR library) is a candidate of end e iff a mate aligns to e with
+ *      S2 and S3; the first such alignment (mate 0 first, + first, smallest d) orients the pair;
+ *   S5-S6 end e's reads: its pairs in ascending pair index, mate 0 then mate 1, each in contig-forward
+ *      orientation (the mate on the - strand reverse-complemented, its qualities reversed).
+ * Input: contigs and a pool of reads as sequenced (la_pool; mem = LA_MEM_HOST or LA_MEM_DEVICE on the
+ * context's device; read length is not limited here).  Output (*out): the selected (end, pair, flip)
+ * records, sorted by (end, pair), flip = 1 when mate 0 is the reverse-complemented one, and `batch`,
+ * an la_batch with mem = LA_MEM_DEVICE that la_load_batch takes directly (its contig arrays are the
+ * library's device copy of the pool's contigs).  All output pointers are device memory owned by the
+ * context, valid until the next la_select_reads or la_destroy on it.  The call runs on the context
+ * stream and returns when the selection is complete.
+ * Errors: LA_ERR_INVALID_ARG for NULL pointers, n_contigs < 0, n_pairs < 0, non-monotone offsets, or
+ * parameters out of range (1 <= seed_len <= 31, seed_stride >= 1, seed_len <= window <= 65535,
+ * min_overlap >= 0, 0 <= max_mism_pct <= 100); LA_ERR_OOM; LA_ERR_CUDA (sticky). */
+typedef struct {
+    int32_t mem;                                          /* LA_MEM_HOST or LA_MEM_DEVICE */
+    int32_t n_contigs;
+    const char *contig_seq; const int64_t *contig_off;    /* [n_contigs+1] */
+    int64_t n_pairs;                                      /* reads 2i, 2i+1 are the mates of pair i */
+    const char *read_seq, *read_qual; const int64_t *read_off;   /* [2*n_pairs+1] */
+} la_pool;
+typedef struct {
+    int32_t window;         /* S1, default 150 */
+    int32_t seed_len;       /* S2(a), default 16 */
+    int32_t seed_stride;    /* S2(a), default 4 */
+    int32_t min_overlap;    /* S2(b), default 20 */
+    int32_t max_mism_pct;   /* S2(c), default 4 */
+} la_sel_params;
+typedef struct {
+    int64_t n_sel;                                        /* selected (end, pair) records */
+    const int64_t *sel_end, *sel_pair;                    /* device [n_sel] */
+    const uint8_t *sel_flip;                              /* device [n_sel] */
+    la_batch batch;                                       /* device; n_reads = 2 * n_sel */
+} la_selection;
+la_status la_select_reads(la_ctx *ctx, const la_pool *pool, const la_sel_params *sp, la_selection *out);
+
 la_status la_get_stats(const la_ctx *ctx, la_stats *out);
 la_status la_destroy(la_ctx *ctx);                /* NULL is a no-op */
 const char *la_last_error(const la_ctx *ctx);     /* message of the last non-OK status */

@@ -61,8 +61,24 @@ class la_stats(ctypes.Structure):
                 ("cpu_attempts", ctypes.c_int64)]
 
 
+class la_pool(ctypes.Structure):
+    _fields_ = [("mem", ctypes.c_int32), ("n_contigs", ctypes.c_int32),
+                ("contig_seq", ctypes.c_void_p), ("contig_off", ctypes.c_void_p),
+                ("n_pairs", ctypes.c_int64),
+                ("read_seq", ctypes.c_void_p), ("read_qual", ctypes.c_void_p), ("read_off", ctypes.c_void_p)]
+
+
+class la_sel_params(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("window", "seed_len", "seed_stride", "min_overlap", "max_mism_pct")]
+
+
+class la_selection(ctypes.Structure):
+    _fields_ = [("n_sel", ctypes.c_int64), ("sel_end", ctypes.c_void_p), ("sel_pair", ctypes.c_void_p),
+                ("sel_flip", ctypes.c_void_p), ("batch", la_batch)]
+
+
 EXPORTS = ["la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
-           "la_replay_build", "la_set_coexec",
+           "la_replay_build", "la_set_coexec", "la_select_reads",
            "la_get_stats", "la_destroy", "la_last_error", "la_plan_global_capacity", "la_paper_load_factor"]
 
 _lib = None
@@ -94,6 +110,8 @@ def load():
     lib.la_get_stats.argtypes = [V, ctypes.POINTER(la_stats)]
     lib.la_replay_build.argtypes = [V]
     lib.la_set_coexec.argtypes = [V, ctypes.c_int32, ctypes.c_double]
+    lib.la_select_reads.argtypes = [V, ctypes.POINTER(la_pool), ctypes.POINTER(la_sel_params),
+                                    ctypes.POINTER(la_selection)]
     lib.la_destroy.argtypes = [V]
     lib.la_last_error.argtypes = [V]
     lib.la_last_error.restype = ctypes.c_char_p
@@ -102,7 +120,7 @@ def load():
     lib.la_paper_load_factor.argtypes = [ctypes.c_int32, ctypes.c_int32]
     lib.la_paper_load_factor.restype = ctypes.c_double
     for f in ("la_create", "la_load_batch", "la_extend", "la_extend_device", "la_extend_streamed", "la_append_extensions",
-              "la_replay_build", "la_set_coexec", "la_get_stats", "la_destroy"):
+              "la_replay_build", "la_set_coexec", "la_select_reads", "la_get_stats", "la_destroy"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib

@@ -188,6 +188,38 @@ class LocalAssembler:
                                                    eoff_ptr, eseq_ptr, out_seq.data_ptr(), out_off.data_ptr()))
         return out_seq[:tot], out_off
 
+    SEL_DEFAULTS = dict(window=150, seed_len=16, seed_stride=4, min_overlap=20, max_mism_pct=4)
+
+    def select_reads(self, pool, **sel):
+        """la_select_reads (NEXT N4): candidate reads of every contig end from a pool of FR read pairs
+        (attributes contig_seq, contig_off, read_seq, read_qual, read_off; reads 2i, 2i+1 are mates),
+        readings S1-S6 of DESIGN.md §10d.  Returns (records, batch): records = dict of host arrays
+        sel_end / sel_pair / sel_flip; batch = a DeviceBatch whose arrays stay on the device (context-owned,
+        valid until the next select_reads) and can be passed to load()."""
+        fields = (("contig_seq", "bytes"), ("contig_off", "int64"), ("read_seq", "bytes"), ("read_qual", "bytes"),
+                  ("read_off", "int64"))
+        arrs = [getattr(pool, f) for f, _ in fields]
+        ptrs, devs, keep = zip(*[_ptr_and_mem(a, f, w, self._device) for a, (f, w) in zip(arrs, fields)])
+        if len(set(devs)) != 1:
+            raise ValueError("pool arrays must all be host or all be device memory")
+        n_reads = int(arrs[4].shape[0]) - 1
+        if n_reads % 2:
+            raise ValueError("read_off must describe an even number of reads (pairs)")
+        pl = L.la_pool(L.LA_MEM_DEVICE if devs[0] else L.LA_MEM_HOST, int(arrs[1].shape[0]) - 1, ptrs[0], ptrs[1],
+                       n_reads // 2, ptrs[2], ptrs[3], ptrs[4])
+        sp = dict(self.SEL_DEFAULTS, **sel)
+        spc = L.la_sel_params(*[int(sp[n]) for n, _ in L.la_sel_params._fields_])
+        out = L.la_selection()
+        self._check(self._lib.la_select_reads(self._ctx, ctypes.byref(pl), ctypes.byref(spc), ctypes.byref(out)))
+        del keep
+        return _selection(out)
+
+    def load_device_batch(self, b, params=None):
+        """la_load_batch on an la_batch struct of device pointers (e.g. select_reads()'s batch)."""
+        p = _params(params)
+        self._check(self._lib.la_load_batch(self._ctx, ctypes.byref(b.raw), ctypes.byref(p)))
+        return self
+
     def set_coexec(self, n_threads: int, cpu_share: float):
         """la_set_coexec: NEXT N3 CPU+GPU co-execution (the lightest ends of the smallest class on host
         threads while the GPU runs); n_threads = 0 turns it off."""
@@ -226,6 +258,51 @@ class LocalAssembler:
             self.close()
         except Exception:
             pass
+
+
+@dataclass
+class DeviceBatch:
+    """An la_batch of context-owned device pointers (select_reads); `host()` copies it to numpy."""
+    raw: object
+    n_contigs: int
+    n_reads: int
+
+    def host(self) -> dict:
+        b = self.raw
+        coff = _d2h(b.contig_off, self.n_contigs + 1, np.int64)
+        roff = _d2h(b.read_off, self.n_reads + 1, np.int64)
+        return dict(contig_off=coff, contig_seq=_d2h(b.contig_seq, int(coff[-1]), np.uint8), read_off=roff,
+                    read_seq=_d2h(b.read_seq, int(roff[-1]), np.uint8),
+                    read_qual=_d2h(b.read_qual, int(roff[-1]), np.uint8),
+                    end_read_off=_d2h(b.end_read_off, 2 * self.n_contigs + 1, np.int64))
+
+
+_CUDART = None
+
+
+def _d2h(ptr, count: int, dtype) -> np.ndarray:
+    """Copy `count` elements at a library-owned device pointer into a new numpy array (cudaMemcpy of the
+    CUDA runtime torch loads; the library's own runtime is linked statically and not exported)."""
+    global _CUDART
+    out = np.zeros(count, dtype)
+    if count == 0:
+        return out
+    if _CUDART is None:
+        import torch   # noqa: F401  (loads libcudart)
+        _CUDART = ctypes.CDLL("libcudart.so.12")
+        _CUDART.cudaMemcpy.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int]
+        _CUDART.cudaMemcpy.restype = ctypes.c_int
+    if _CUDART.cudaMemcpy(out.ctypes.data, ctypes.c_void_p(ptr), out.nbytes, 2) != 0:   # cudaMemcpyDeviceToHost
+        raise RuntimeError("cudaMemcpy (device to host) failed")
+    return out
+
+
+def _selection(out):
+    n = int(out.n_sel)
+    rec = dict(sel_end=_d2h(out.sel_end, n, np.int64), sel_pair=_d2h(out.sel_pair, n, np.int64),
+               sel_flip=_d2h(out.sel_flip, n, np.uint8))
+    b = out.batch
+    return rec, DeviceBatch(b, int(b.n_contigs), int(b.n_reads))
 
 
 def extend(batch, params=None, device: int = 0) -> Result:

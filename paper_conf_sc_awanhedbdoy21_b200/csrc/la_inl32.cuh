@@ -28,6 +28,17 @@
 #endif
 namespace la {
 
+#ifdef LA_PROBE_STATS
+// debug build only (tools/probe_stats.py): [0] warp_insert32 calls (per warp), [1] their probe rounds,
+// [2] inserting lanes, [3] claims, [4] warp_lookup32 calls, [5] their rounds, [6] looking-up lanes,
+// [7] unused, [8] filter-pass warp iterations, [9] their voting lanes, [10] 128-bit CAS issued,
+// [11] slot re-reads after a racing claim
+__device__ unsigned long long g_probe_stats[12];
+#define LA_PSTAT(i, v) atomicAdd(&g_probe_stats[i], (unsigned long long)(v))
+#else
+#define LA_PSTAT(i, v) ((void)0)
+#endif
+
 template <int NW>
 struct K32 {
     uint32_t w[NW];
@@ -254,6 +265,7 @@ __device__ __forceinline__ int cmp_slot(const Tab32 &T, uint32_t s, uint4 v, con
     if (v.w == 0u) return 2;
     if (v.w != f.w) return 1;
     if (v.x == f.x && v.y == f.y && v.z == f.z) return 0;
+    LA_PSTAT(11, 1);
     v = ld_slot<GT>(T, s);
     return (v.x == f.x && v.y == f.y && v.z == f.z) ? 0 : 1;
 }
@@ -267,7 +279,14 @@ __device__ __forceinline__ void warp_insert32(const Tab32 &T, bool want, const u
                                               uint32_t &vpend) {
     uint32_t s = slot32(h, T.cap), hit = 0;
     bool pend = want, found = false;
+#ifdef LA_PROBE_STATS
+    {
+        const unsigned wm = __ballot_sync(0xffffffffu, want);
+        if (lane == 0) { LA_PSTAT(0, 1); LA_PSTAT(2, __popc(wm)); }
+    }
+#endif
     while (__any_sync(0xffffffffu, pend)) {
+        if (lane == 0) LA_PSTAT(1, 1);
         bool claimed = false;
         if (pend) {
             const uint32_t s1 = s + 1;   // s even, cap even
@@ -286,6 +305,7 @@ __device__ __forceinline__ void warp_insert32(const Tab32 &T, bool want, const u
                 if (*ovf) {
                     pend = false;
                 } else {
+                    LA_PSTAT(10, 1);
                     const uint4 o = cas_slot<GT>(T, at, f);
                     if (o.w == 0u) {
                         claimed = found = true;
@@ -313,6 +333,7 @@ __device__ __forceinline__ void warp_insert32(const Tab32 &T, bool want, const u
                 s = s1 + 1 == T.cap ? 0 : s1 + 1;
             }
         }
+        if (claimed) LA_PSTAT(3, 1);
         if (claimed) {   // claim list: one shared atomic per claim (claims <= cap: no overflow)
             const int idx = LA_ABL_NOCLAIM ? (int)(hit & 1023u) : atomicAdd(nclaim, 1);
             if (idx >= claim_limit) *ovf = 1;
@@ -327,7 +348,14 @@ template <bool GT>
 __device__ __forceinline__ uint32_t warp_lookup32(const Tab32 &T, bool want, const uint4 f, uint32_t h) {
     uint32_t s = slot32(h, T.cap), res = NONE, n = 0;
     bool pend = want;
+#ifdef LA_PROBE_STATS
+    {
+        const unsigned wm = __ballot_sync(0xffffffffu, want);
+        if ((threadIdx.x & 31) == 0) { LA_PSTAT(4, 1); LA_PSTAT(6, __popc(wm)); }
+    }
+#endif
     while (__any_sync(0xffffffffu, pend)) {
+        if ((threadIdx.x & 31) == 0) LA_PSTAT(5, 1);
         if (pend) {
             const uint4 v0 = ld_slot<GT>(T, s), v1 = ld_slot<GT>(T, s + 1);
             const int a = cmp_slot<GT>(T, s, v0, f);

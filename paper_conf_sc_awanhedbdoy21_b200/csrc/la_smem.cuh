@@ -491,14 +491,6 @@ __device__ __forceinline__ uint32_t tab_lookup(const TabCtx &T, const KmerN<NW> 
     return NONE;
 }
 
-#ifdef LA_PROBE_STATS
-// debug build only: [0] warp_insert calls, [1] probe rounds, [2] inserting lanes, [3] claims,
-// [4] lookup calls, [5] lookup rounds, [6] looking-up lanes, [7] sum of table loads at link (claims*1000/cap)
-__device__ unsigned long long g_probe_stats[8];
-#define LA_PSTAT(i, v) atomicAdd(&g_probe_stats[i], (unsigned long long)(v))
-#else
-#define LA_PSTAT(i, v) ((void)0)
-#endif
 
 // ---- warp-convergent passes for pointer keys (k >= 64) ----------------------------------------
 __device__ __forceinline__ uint64_t nmask_word(uint64_t q) { return q & (q >> 1) & 0x5555555555555555ull; }
@@ -840,6 +832,12 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
         if (mbits) {
             // ---- filter pass: B1 = seen once, B2 = seen at least twice (reading #4) ----
             auto filt = [&](bool, bool act, uint32_t, const K32<NW> &, uint32_t h, uint32_t, bool) {
+#ifdef LA_PROBE_STATS
+                                     {
+                                         const unsigned am = __ballot_sync(0xffffffffu, act);
+                                         if (lane == 0) { LA_PSTAT(8, 1); LA_PSTAT(9, __popc(am)); }
+                                     }
+#endif
                                      if (!act) return;
                                      const uint32_t fi = filt32(h, mbits);
                                      const uint32_t bit = 1u << (fi & 31);

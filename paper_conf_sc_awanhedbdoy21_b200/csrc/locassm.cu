@@ -17,6 +17,7 @@
 #include "locassm.h"
 #include "la_cpu.h"
 #include "la_kernels.cuh"
+#include "la_select.cuh"
 
 using namespace la;
 
@@ -39,6 +40,18 @@ struct HostBuf {
         if (p) cudaFreeHost(p);
         p = nullptr;
         n = 0;
+    }
+};
+
+// NEXT N4 (la_select_reads): device copies of the pool and the selection's scratch and results.
+struct SelBufs {
+    DevBuf cseq, coff, rseq, rqual, roff, wcnt, woff, key, val, key2, val2, flag, uidx, ustart, hkey, hval, nrec,
+        rkey, rord, rkey2, rord2, send, spair, sflip, eoff, lens, ooff, oseq, oqual;
+    void release() {
+        for (DevBuf *b : {&cseq, &coff, &rseq, &rqual, &roff, &wcnt, &woff, &key, &val, &key2, &val2, &flag, &uidx,
+                          &ustart, &hkey, &hval, &nrec, &rkey, &rord, &rkey2, &rord2, &send, &spair, &sflip, &eoff,
+                          &lens, &ooff, &oseq, &oqual})
+            b->release();
     }
 };
 
@@ -140,6 +153,7 @@ struct la_ctx {
     // fills the GPU, so only their tails can overlap) while making the per-class times overlapping
     // spans; LA_CONCURRENT_CLASSES=1 restores the concurrent launch.
     bool concurrent_classes = false;
+    SelBufs sel;   // NEXT N4
     la_stats stats{};
 };
 
@@ -347,6 +361,7 @@ extern "C" la_status la_destroy(la_ctx *ctx) {
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     ctx->enc.release();
     ctx->spare.release();
+    ctx->sel.release();
     for (int i = 0; i < 2; ++i) {
         for (DevBuf *b : {&ctx->st_seq[i], &ctx->st_qual[i], &ctx->st_cseq[i], &ctx->st_coff[i], &ctx->st_roff[i],
                           &ctx->st_eoff[i]})
@@ -401,9 +416,9 @@ extern "C" la_status la_get_stats(const la_ctx *ctx, la_stats *out) {
 extern "C" int64_t la_plan_global_capacity(int64_t inserts) { return global_capacity(inserts); }
 #ifdef LA_PROBE_STATS
 extern "C" int la_debug_probe_stats(unsigned long long *out, int reset) {
-    if (cudaMemcpyFromSymbol(out, g_probe_stats, sizeof(unsigned long long) * 8) != cudaSuccess) return -1;
+    if (cudaMemcpyFromSymbol(out, g_probe_stats, sizeof(unsigned long long) * 12) != cudaSuccess) return -1;
     if (reset) {
-        unsigned long long z[8] = {};
+        unsigned long long z[12] = {};
         cudaMemcpyToSymbol(g_probe_stats, z, sizeof(z));
     }
     return 0;
@@ -1429,5 +1444,214 @@ extern "C" la_status la_append_extensions(la_ctx *ctx, int32_t n_contigs, const 
                                                        out_off);
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(ctx->stream));
+    return LA_OK;
+}
+
+// ================================================================================================
+// NEXT N4: la_select_reads — candidate-read selection on the device (la_select.cuh)
+// ================================================================================================
+namespace {
+
+template <typename T>
+la_status cub_scan(la_ctx *ctx, const T *in, T *out, int64_t n) {
+    size_t tb = 0;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, in, out, n, ctx->stream));
+    CK(grow(ctx->cub_tmp, tb));
+    CK(cub::DeviceScan::ExclusiveSum(ctx->cub_tmp.p, tb, in, out, n, ctx->stream));
+    return LA_OK;
+}
+
+template <typename K, typename V>
+la_status cub_sort_pairs(la_ctx *ctx, const K *kin, K *kout, const V *vin, V *vout, int64_t n) {
+    size_t tb = 0;
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, kin, kout, vin, vout, n, 0, (int)(8 * sizeof(K)), ctx->stream));
+    CK(grow(ctx->cub_tmp, tb));
+    CK(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp.p, tb, kin, kout, vin, vout, n, 0, (int)(8 * sizeof(K)),
+                                       ctx->stream));
+    return LA_OK;
+}
+
+la_status d2h_i64(la_ctx *ctx, const int64_t *d, int64_t *h) {
+    CK(cudaMemcpyAsync(h, d, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return LA_OK;
+}
+
+}  // namespace
+
+extern "C" la_status la_select_reads(la_ctx *ctx, const la_pool *pool, const la_sel_params *sp, la_selection *out) {
+    if (!ctx) return LA_ERR_INVALID_ARG;
+    if (ctx->sticky) return fail(ctx, LA_ERR_CUDA, "context has a sticky CUDA error: %s", ctx->err.c_str());
+    if (!pool || !sp || !out) return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: null argument");
+    if (pool->n_contigs < 0 || pool->n_pairs < 0 || pool->n_pairs > 0xFFFFFFFFll)
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: n_contigs or n_pairs out of range");
+    if (!pool->contig_off || !pool->read_off || (pool->n_pairs && (!pool->read_seq || !pool->read_qual)) ||
+        (pool->n_contigs && !pool->contig_seq))
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: null pool array");
+    if (pool->mem != LA_MEM_HOST && pool->mem != LA_MEM_DEVICE)
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: mem must be LA_MEM_HOST or LA_MEM_DEVICE");
+    if (!(sp->seed_len >= 1 && sp->seed_len <= 31 && sp->seed_stride >= 1 && sp->window >= sp->seed_len &&
+          sp->window <= 65535 && sp->min_overlap >= 0 && sp->max_mism_pct >= 0 && sp->max_mism_pct <= 100))
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: parameters out of range");
+    CK(cudaSetDevice(ctx->device));
+    cudaStream_t st = ctx->stream;
+    SelBufs &S = ctx->sel;
+    const bool host = pool->mem == LA_MEM_HOST;
+    const int64_t nC = pool->n_contigs, nE = 2 * nC, nR = 2 * pool->n_pairs;
+    // ---- input: offsets validated (monotone, starting at 0), arrays copied to the device ----
+    int64_t c0, cN, r0, rN;
+    la_status rc;
+    if ((rc = read_i64(ctx, pool->contig_off, host, &c0)) != LA_OK) return rc;
+    if ((rc = read_i64(ctx, pool->contig_off + nC, host, &cN)) != LA_OK) return rc;
+    if ((rc = read_i64(ctx, pool->read_off, host, &r0)) != LA_OK) return rc;
+    if ((rc = read_i64(ctx, pool->read_off + nR, host, &rN)) != LA_OK) return rc;
+    if (c0 != 0 || r0 != 0 || cN < 0 || rN < 0)
+        return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: offsets must start at 0 and be non-decreasing");
+    if ((rc = copy_in(ctx, S.coff, pool->contig_off, 8 * (size_t)(nC + 1), host)) != LA_OK) return rc;
+    if ((rc = copy_in(ctx, S.roff, pool->read_off, 8 * (size_t)(nR + 1), host)) != LA_OK) return rc;
+    if ((rc = copy_in(ctx, S.cseq, pool->contig_seq, (size_t)cN, host)) != LA_OK) return rc;
+    if ((rc = copy_in(ctx, S.rseq, pool->read_seq, (size_t)rN, host)) != LA_OK) return rc;
+    if ((rc = copy_in(ctx, S.rqual, pool->read_qual, (size_t)rN, host)) != LA_OK) return rc;
+    CK(grow(ctx->errw, 16));
+    uint32_t *d_err = P<uint32_t>(ctx->errw);
+    CK(cudaMemsetAsync(d_err, 0, 4, st));
+    if (nC) { k_check_offsets<<<blocks(nC, 256), 256, 0, st>>>(P<int64_t>(S.coff), nC, 0, d_err, nullptr); CKL(); }
+    if (nR) { k_check_offsets<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(S.roff), nR, 0, d_err, nullptr); CKL(); }
+    uint32_t h_err = 0;
+    CK(cudaMemcpyAsync(&h_err, d_err, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (h_err) return fail(ctx, LA_ERR_INVALID_ARG, "la_select_reads: offsets are not non-decreasing");
+    const int w = sp->window, s = sp->seed_len, t = sp->seed_stride;
+    // ---- index of the end windows' seeds (S1, S2a) ----
+    CK(grow(S.wcnt, 8 * (size_t)(nE + 1)));
+    CK(grow(S.woff, 8 * (size_t)(nE + 1)));
+    CK(cudaMemsetAsync(S.wcnt.p, 0, 8 * (size_t)(nE + 1), st));
+    if (nE) { sel::k_sel_wcount<<<blocks(nE, 256), 256, 0, st>>>(nE, P<int64_t>(S.coff), w, s, P<int64_t>(S.wcnt)); CKL(); }
+    if ((rc = cub_scan(ctx, P<int64_t>(S.wcnt), P<int64_t>(S.woff), nE + 1)) != LA_OK) return rc;
+    int64_t nI = 0;
+    if ((rc = d2h_i64(ctx, P<int64_t>(S.woff) + nE, &nI)) != LA_OK) return rc;
+    int64_t nU = 0;
+    uint64_t cap_mask = 0;
+    if (nI) {
+        for (DevBuf *b : {&S.key, &S.val, &S.key2, &S.val2}) CK(grow(*b, 8 * (size_t)nI));
+        CK(grow(S.flag, 8 * (size_t)(nI + 1)));
+        CK(grow(S.uidx, 8 * (size_t)(nI + 1)));
+        sel::k_sel_index<<<blocks(32 * nE, 256), 256, 0, st>>>(nE, P<char>(S.cseq), P<int64_t>(S.coff), P<int64_t>(S.woff),
+                                                                w, s, P<uint64_t>(S.key), P<uint64_t>(S.val));
+        CKL();
+        if ((rc = cub_sort_pairs(ctx, P<uint64_t>(S.key), P<uint64_t>(S.key2), P<uint64_t>(S.val), P<uint64_t>(S.val2),
+                                 nI)) != LA_OK)
+            return rc;
+        CK(cudaMemsetAsync(P<int64_t>(S.flag) + nI, 0, 8, st));
+        sel::k_sel_runs<<<blocks(nI, 256), 256, 0, st>>>(nI, P<uint64_t>(S.key2), P<int64_t>(S.flag));
+        CKL();
+        if ((rc = cub_scan(ctx, P<int64_t>(S.flag), P<int64_t>(S.uidx), nI + 1)) != LA_OK) return rc;
+        if ((rc = d2h_i64(ctx, P<int64_t>(S.uidx) + nI, &nU)) != LA_OK) return rc;
+    }
+    {
+        uint64_t cap = 1024;
+        while (cap < 2 * (uint64_t)nU) cap <<= 1;
+        cap_mask = cap - 1;
+        CK(grow(S.hkey, 8 * cap));
+        CK(grow(S.hval, 8 * cap));
+        CK(grow(S.ustart, 8 * (size_t)(nU + 1)));
+        CK(cudaMemsetAsync(S.hkey.p, 0, 8 * cap, st));
+        CK(cudaMemsetAsync(S.ustart.p, 0, 8 * (size_t)(nU + 1), st));
+        if (nU) {
+            sel::k_sel_hash<<<blocks(nI, 256), 256, 0, st>>>(nI, P<uint64_t>(S.key2), P<int64_t>(S.flag), P<int64_t>(S.uidx),
+                                                              P<int64_t>(S.ustart), cap_mask,
+                                                              P<unsigned long long>(S.hkey), P<int64_t>(S.hval));
+            CKL();
+            // ustart[nU] = number of valid entries (KEY_NONE sorts last): the last run ends there
+            sel::k_sel_nvalid<<<blocks(nI, 256), 256, 0, st>>>(nI, P<uint64_t>(S.key2), P<int64_t>(S.ustart) + nU);
+            CKL();
+        }
+    }
+    // ---- queries (S2, S3): records of qualifying alignments; regrown and rerun if they overflow ----
+    CK(grow(S.nrec, 8));
+    int64_t cap_rec = std::max<int64_t>(1024, 2 * nR);
+    int64_t n_rec = 0;
+    for (int pass = 0; pass < 8; ++pass) {
+        for (DevBuf *b : {&S.rkey, &S.rkey2}) CK(grow(*b, 8 * (size_t)cap_rec));
+        for (DevBuf *b : {&S.rord, &S.rord2}) CK(grow(*b, 4 * (size_t)cap_rec));
+        CK(cudaMemsetAsync(S.nrec.p, 0, 8, st));
+        if (nR && nU) {
+            sel::k_sel_query<<<blocks(2 * nR, 128), 128, 0, st>>>(
+                nR / 2 * 2, P<char>(S.rseq), P<int64_t>(S.roff), P<char>(S.cseq), P<int64_t>(S.coff), w, s, t,
+                sp->min_overlap, sp->max_mism_pct, P<unsigned long long>(S.hkey), P<int64_t>(S.hval), cap_mask,
+                P<int64_t>(S.ustart), P<uint64_t>(S.val2), P<unsigned long long>(S.nrec), cap_rec, P<uint64_t>(S.rkey),
+                P<uint32_t>(S.rord));
+            CKL();
+        }
+        if ((rc = d2h_i64(ctx, P<int64_t>(S.nrec), &n_rec)) != LA_OK) return rc;
+        if (n_rec <= cap_rec) break;
+        cap_rec = n_rec + n_rec / 4 + 1024;
+        if (pass == 7) return fail(ctx, LA_ERR_CAPACITY, "la_select_reads: record buffer did not converge");
+    }
+    // ---- S4: sort records by (end, pair), then (mate, strand, d); keep the first of each (end, pair) ----
+    int64_t n_sel = 0;
+    if (n_rec) {
+        // stable radix sorts: by ord first (carrying the key), then by key (carrying the ord)
+        if ((rc = cub_sort_pairs(ctx, P<uint32_t>(S.rord), P<uint32_t>(S.rord2), P<uint64_t>(S.rkey), P<uint64_t>(S.rkey2),
+                                 n_rec)) != LA_OK)
+            return rc;
+        if ((rc = cub_sort_pairs(ctx, P<uint64_t>(S.rkey2), P<uint64_t>(S.rkey), P<uint32_t>(S.rord2), P<uint32_t>(S.rord),
+                                 n_rec)) != LA_OK)
+            return rc;
+        CK(grow(S.flag, 8 * (size_t)(n_rec + 1)));
+        CK(grow(S.uidx, 8 * (size_t)(n_rec + 1)));
+        CK(cudaMemsetAsync(P<int64_t>(S.flag) + n_rec, 0, 8, st));
+        sel::k_sel_first<<<blocks(n_rec, 256), 256, 0, st>>>(n_rec, P<uint64_t>(S.rkey), P<int64_t>(S.flag));
+        CKL();
+        if ((rc = cub_scan(ctx, P<int64_t>(S.flag), P<int64_t>(S.uidx), n_rec + 1)) != LA_OK) return rc;
+        if ((rc = d2h_i64(ctx, P<int64_t>(S.uidx) + n_rec, &n_sel)) != LA_OK) return rc;
+    }
+    CK(grow(S.send, 8 * (size_t)(n_sel + 1)));
+    CK(grow(S.spair, 8 * (size_t)(n_sel + 1)));
+    CK(grow(S.sflip, (size_t)(n_sel + 1)));
+    if (n_sel) {
+        sel::k_sel_compact<<<blocks(n_rec, 256), 256, 0, st>>>(n_rec, P<uint64_t>(S.rkey), P<uint32_t>(S.rord),
+                                                                P<int64_t>(S.flag), P<int64_t>(S.uidx), P<int64_t>(S.send),
+                                                                P<int64_t>(S.spair), P<uint8_t>(S.sflip));
+        CKL();
+    }
+    // ---- S5-S6: the batch ----
+    const int64_t nOut = 2 * n_sel;
+    CK(grow(S.eoff, 8 * (size_t)(nE + 1)));
+    CK(grow(S.lens, 8 * (size_t)(nOut + 1)));
+    CK(grow(S.ooff, 8 * (size_t)(nOut + 1)));
+    sel::k_sel_eoff<<<blocks(nE + 1, 256), 256, 0, st>>>(nE, n_sel, P<int64_t>(S.send), P<int64_t>(S.eoff));
+    CKL();
+    CK(cudaMemsetAsync(P<int64_t>(S.lens) + nOut, 0, 8, st));
+    if (nOut) {
+        sel::k_sel_lens<<<blocks(nOut, 256), 256, 0, st>>>(n_sel, P<int64_t>(S.spair), P<int64_t>(S.roff), P<int64_t>(S.lens));
+        CKL();
+    }
+    if ((rc = cub_scan(ctx, P<int64_t>(S.lens), P<int64_t>(S.ooff), nOut + 1)) != LA_OK) return rc;
+    int64_t out_bytes = 0;
+    if ((rc = d2h_i64(ctx, P<int64_t>(S.ooff) + nOut, &out_bytes)) != LA_OK) return rc;
+    CK(grow(S.oseq, (size_t)out_bytes + 16));
+    CK(grow(S.oqual, (size_t)out_bytes + 16));
+    if (nOut) {
+        sel::k_sel_copy<<<blocks(32 * nOut, 256), 256, 0, st>>>(n_sel, P<int64_t>(S.spair), P<uint8_t>(S.sflip), P<char>(S.rseq),
+                                                                 P<char>(S.rqual), P<int64_t>(S.roff), P<int64_t>(S.ooff),
+                                                                 P<char>(S.oseq), P<char>(S.oqual));
+        CKL();
+    }
+    CK(cudaStreamSynchronize(st));
+    out->n_sel = n_sel;
+    out->sel_end = P<int64_t>(S.send);
+    out->sel_pair = P<int64_t>(S.spair);
+    out->sel_flip = P<uint8_t>(S.sflip);
+    la_batch &B = out->batch;
+    B.mem = LA_MEM_DEVICE;
+    B.n_contigs = (int32_t)nC;
+    B.contig_seq = P<char>(S.cseq);
+    B.contig_off = P<int64_t>(S.coff);
+    B.n_reads = nOut;
+    B.read_seq = P<char>(S.oseq);
+    B.read_qual = P<char>(S.oqual);
+    B.read_off = P<int64_t>(S.ooff);
+    B.end_read_off = P<int64_t>(S.eoff);
     return LA_OK;
 }

@@ -202,3 +202,106 @@ def test_select_reverse_complement_symmetry(orc):
         m = ia[(e ^ 1, p)]
         for mate in (0, 1):
             assert sb[ob[2 * n + mate]:ob[2 * n + mate + 1]] == _rc(sa[oa[2 * m + mate]:oa[2 * m + mate + 1]])
+
+
+# ---------------------------------------------------------------------------------------------- GPU
+
+def _gpu_select(pool, **kw):
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    la = LocalAssembler(0)
+    rec, db = la.select_reads(pool, **dict(GPU_SP, **kw))
+    return la, rec, db
+
+
+def _check_same(orc_r, rec, host):
+    for f in ("sel_end", "sel_pair", "sel_flip"):
+        assert np.array_equal(rec[f], orc_r[f]), f
+    for f in ("end_read_off", "read_off", "read_seq", "read_qual"):
+        assert np.array_equal(host[f], orc_r[f]), f
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("kind", ["error_free", "errors_repeats_N", "short_contigs"])
+def test_gpu_select_matches_oracle(orc, kind):
+    if kind == "error_free":
+        pool = make_pool(seed=7, genome_len=30000, n_contigs=14, coverage=12, err=0.0, n_rate=0.0, unique_k=16)
+    elif kind == "errors_repeats_N":
+        pool = make_pool(seed=31, genome_len=80000, n_contigs=50, coverage=25, err=0.015, n_rate=2e-3, repeats=6)
+    else:
+        pool = make_pool(seed=32, genome_len=20000, n_contigs=25, contig_len=(10, 300), coverage=20)
+    r = _select(orc, pool)
+    la, rec, db = _gpu_select(pool)
+    try:
+        _check_same(r, rec, db.host())
+    finally:
+        la.close()
+    assert kind == "short_contigs" or rec["sel_end"].size > 100
+
+
+@pytest.mark.gpu
+def test_gpu_select_parameters_and_device_input(orc):
+    import torch
+    pool = make_pool(seed=33, genome_len=40000, n_contigs=20, coverage=20, err=0.02, n_rate=1e-3, repeats=4)
+    for kw in (dict(w=100, s=12, t=1, o=12, mm_pct=0), dict(w=300, s=31, t=7, o=40, mm_pct=10)):
+        r = _select(orc, pool, **kw)
+        gkw = dict(window=kw["w"], seed_len=kw["s"], seed_stride=kw["t"], min_overlap=kw["o"], max_mism_pct=kw["mm_pct"])
+        la, rec, db = _gpu_select(pool, **gkw)
+        _check_same(r, rec, db.host())
+        la.close()
+    # device-memory pool (torch CUDA tensors)
+
+    class D:
+        pass
+    d = D()
+    for f in ("contig_seq", "contig_off", "read_seq", "read_qual", "read_off"):
+        setattr(d, f, torch.from_numpy(getattr(pool, f)).cuda())
+    r = _select(orc, pool)
+    la, rec, db = _gpu_select(d)
+    _check_same(r, rec, db.host())
+    la.close()
+
+
+@pytest.mark.gpu
+def test_gpu_select_degenerate_and_invalid():
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    from paper_conf_sc_awanhedbdoy21_b200._lib import LocAssmError
+
+    class P:
+        pass
+    p = P()
+    p.contig_seq = np.frombuffer(b"ACGT" * 50, np.uint8).copy()
+    p.contig_off = np.array([0, 200], np.int64)
+    p.read_seq = np.zeros(0, np.uint8)
+    p.read_qual = np.zeros(0, np.uint8)
+    p.read_off = np.zeros(1, np.int64)
+    with LocalAssembler(0) as la:
+        rec, db = la.select_reads(p)
+        assert rec["sel_end"].size == 0
+        assert np.array_equal(db.host()["end_read_off"], np.zeros(3, np.int64))
+        p.contig_off = np.array([0, 250], np.int64)[::-1].copy()
+        with pytest.raises(LocAssmError):
+            la.select_reads(p)
+        p.contig_off = np.array([0, 200], np.int64)
+        with pytest.raises(LocAssmError):
+            la.select_reads(p, seed_len=40)
+
+
+@pytest.mark.gpu
+def test_gpu_select_then_extend_matches_oracle(orc):
+    """N4 -> local assembly on the device: la_select_reads' batch goes straight into la_load_batch
+    (LA_MEM_DEVICE) and la_extend; the oracle extends the oracle's selection of the same pool."""
+    from gen import Batch, Params
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    pool = make_pool(seed=34, genome_len=120000, n_contigs=60, coverage=30, err=0.01, n_rate=1e-4, repeats=4)
+    r = _select(orc, pool)
+    qual = r["read_qual"].copy()
+    b = Batch(pool.contig_seq, pool.contig_off, r["read_seq"], qual, r["read_off"], r["end_read_off"])
+    ref = orc.extend(b, Params())
+    with LocalAssembler(0) as la:
+        rec, db = la.select_reads(pool, **GPU_SP)
+        la.load_device_batch(db, Params())
+        res = la.extend()
+    assert res.ext_list() == ref["ext"]
+    for f in ("term", "k_used", "n_attempts"):
+        assert np.array_equal(getattr(res, f), ref[f]), f
+    assert sum(len(x) for x in ref["ext"]) > 1000

@@ -29,7 +29,7 @@ def main():
     from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
     lib = ctypes.CDLL(so)
     batch, params = bench.load_workload(a.config, 0, a.scale)
-    out = (ctypes.c_ulonglong * 8)()
+    out = (ctypes.c_ulonglong * 12)()
     res = {}
     for cls in ["64x12,128x6,256x3,256x2,512x1"]:
         with LocalAssembler(0) as la:
@@ -43,7 +43,9 @@ def main():
                     "inserting_lanes_per_call": v[2] / max(v[0], 1), "claims": v[3],
                     "lookup_calls": v[4], "lookup_rounds_per_call": v[5] / max(v[4], 1),
                     "lookup_lanes_per_call": v[6] / max(v[4], 1),
-                    "mean_load_at_link": v[7] / 1000 / max(st["attempts"], 1), "inserts": st["inserts"]}
+                    "filter_warp_iters": v[8], "filter_lanes_per_iter": v[9] / max(v[8], 1),
+                    "cas_issued": v[10], "rereads": v[11], "inserts": st["inserts"],
+                    "ms_total": st["ms_total"]}
     print(json.dumps(res, indent=1))
 
 
