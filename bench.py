@@ -368,6 +368,7 @@ def main():
                     help="minimum number of oracle-checked ends (capped by the batch)")
     ap.add_argument("--no-cpu-baseline", action="store_true", help="skip the oracle (timing and parity)")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-select", action="store_true", help="skip the NEXT N4 selection block")
     ap.add_argument("--no-replay", action="store_true", help="skip the build-only replay (roofline_build)")
     ap.add_argument("--e2e-chunks", type=int, default=8)
     ap.add_argument("--coexec-share", type=float, default=0.05,
@@ -508,6 +509,12 @@ def main():
     del dev
     torch.cuda.empty_cache()
 
+    # ---------------- NEXT N4: candidate-read selection (not part of the step) ----------------
+    select_n4 = None
+    if not args.no_select and rank == 0:
+        select_n4 = bench_select(dev_i, stream)
+        torch.cuda.empty_cache()
+
     # ---------------- end to end through the public API (host buffers) ----------------
     e2e = None
     if not args.no_e2e:
@@ -616,6 +623,7 @@ def main():
         "parity": parity,
         "append_n1": dict(append_n1, peak=peaks["hbm_gbs"], frac=append_n1["achieved"] / peaks["hbm_gbs"]),
         "coexec_n3": n3,
+        "select_n4": select_n4,
         "paper": PAPER,
     }
     if cpu:
@@ -625,7 +633,67 @@ def main():
         log(f"[bench] PARITY FAILURE: {parity['mismatches']} of {parity['ends_checked']} sampled ends differ "
             f"from the oracle: {parity.get('first_mismatch')}")
         return 1
+    if select_n4 and select_n4.get("parity", {}).get("arrays_differing", 0):
+        log(f"[bench] N4 PARITY FAILURE: {select_n4['parity']}")
+        return 1
     return 0
+
+
+def bench_select(dev_i, stream):
+    """NEXT N4 (la_select_reads): candidate-read selection from a pool of FR pairs held in
+    device memory — an 8 Mbp genome, 4000 contigs, 20x coverage (~1.07 M reads), 1% errors; CUDA events
+    around the call (median of 3 after a warm-up).  Parity: the same call on a 60-contig pool against the
+    oracle (oracle/select.cpp), record by record and byte by byte."""
+    import torch
+    from gen.pool import make_pool
+    from paper_conf_sc_awanhedbdoy21_b200 import LocalAssembler
+    sp = dict(window=150, seed_len=16, seed_stride=4, min_overlap=20, max_mism_pct=4)
+    t0 = time.perf_counter()
+    pool = make_pool(seed=20211120, genome_len=8_000_000, n_contigs=4000, contig_len=(400, 3000), coverage=20.0,
+                     err=0.01, n_rate=1e-4, repeats=20)
+    gen_s = time.perf_counter() - t0
+
+    class Dev:
+        pass
+    dp = Dev()
+    for f in ("contig_seq", "contig_off", "read_seq", "read_qual", "read_off"):
+        setattr(dp, f, torch.from_numpy(getattr(pool, f)).cuda(dev_i))
+    ms = []
+    with LocalAssembler(dev_i, stream=stream) as la:
+        for i in range(4):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            rec, db = la.select_reads(dp, **sp)
+            a1.record(stream)
+            a1.synchronize()
+            if i:
+                ms.append(a0.elapsed_time(a1))
+        n_sel = int(rec["sel_end"].size)
+        ends_with = int(np.unique(rec["sel_end"]).size)
+    med = statistics.median(ms)
+    n_reads = 2 * pool.n_pairs
+    out = {"api": "la_select_reads (device pool)", "pool_reads": n_reads, "pool_pairs": pool.n_pairs,
+           "contigs": pool.n_contigs, "genome_bp": 8_000_000, "coverage": 20.0, "pairs_selected": n_sel,
+           "ends_with_reads": ends_with, "ms": med, "value": n_reads / (med / 1e3), "unit": "pool reads/s",
+           "params": sp, "gen_s": round(gen_s, 1),
+           "note": "NEXT N4, outside the timed step; the synchronous call includes its host round trips for "
+                   "buffer sizing (DESIGN.md §10d)"}
+    try:
+        import oracle
+        small = make_pool(seed=20211121, genome_len=60000, n_contigs=60, coverage=25, err=0.015, n_rate=2e-3,
+                          repeats=6)
+        ref = oracle.select_reads(small.contig_seq, small.contig_off, small.read_seq, small.read_qual,
+                                  small.read_off, w=150, s=16, t=4, o=20, mm_pct=4)
+        with LocalAssembler(dev_i, stream=stream) as la:
+            rec, db = la.select_reads(small, **sp)
+            h = db.host()
+        bad = sum(int(not np.array_equal(rec[f], ref[f])) for f in ("sel_end", "sel_pair", "sel_flip")) + \
+            sum(int(not np.array_equal(h[f], ref[f])) for f in ("end_read_off", "read_off", "read_seq", "read_qual"))
+        out["parity"] = {"pairs_checked": int(ref["sel_end"].size), "arrays_differing": bad,
+                         "reference": "oracle/select.cpp on a 60-contig, 10k-pair pool"}
+    except Exception as ex:   # pragma: no cover
+        out["parity"] = {"error": repr(ex)}
+    return out
 
 
 def build_roofline(replay, peaks):

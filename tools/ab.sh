@@ -3,7 +3,7 @@
 # bench per variant on the same GPU box, kernel path only.
 #   gpurun -- bash tools/ab.sh name1 "name2:ENV=1,ENV2=x" ...
 mkdir -p gpurun_out
-python bench.py --config ${CFG:-C4S} --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-replay > /dev/null 2>&1
+timeout 400 python bench.py --config ${CFG:-C4S} --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-replay --no-select --coexec-share 0 > /dev/null 2>&1
 i=0
 for rep in $(seq 1 ${REPS:-2}); do
 for spec in "$@"; do
@@ -11,7 +11,7 @@ for spec in "$@"; do
   v=${spec%%:*}; envs=""; [[ "$spec" == *:* ]] && envs=${spec#*:}
   tag=$(echo "$spec" | tr -c 'A-Za-z0-9_\n' '_')
   ( IFS=','; for kv in $envs; do export "$kv"; done
-    LA_SO=$PWD/build_ab/$v.so LA_SERIAL_CLASSES=${SERIAL:-1} timeout 600 python bench.py --config ${CFG:-C4S} --steps ${STEPS:-5} --warmup 2 \
+    LA_SO=$PWD/build_ab/$v.so LA_SERIAL_CLASSES=${SERIAL:-1} timeout ${RUN_TIMEOUT:-300} python bench.py --config ${CFG:-C4S} --steps ${STEPS:-5} --warmup 2 \
       --no-e2e --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/ab_${tag}_${rep}.json 2> gpurun_out/ab_${tag}_${rep}.err )
   python - "$tag" "$rep" <<'PY'
 import json, sys
