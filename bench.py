@@ -47,6 +47,7 @@ CONFIG_DESC = {
     "C3": "C3 high-skew (18 ends with >40k reads + ~60k sparse ends)",
     "C4": "C4 paper-shaped batch (500-species metagenome, lognormal(0,1.5), 150 bp pairs, ~1M contigs) on 1 B200",
     "C4S": "C4S = r01's C4 (500-species metagenome, 510k contigs, 31.7M read copies)",
+    "C4F": "C4F = C4's contigs with the paper's Fig 3 mix of reads per end (70% none, 29% 1-9, 1% all)",
 }
 CACHE = os.environ.get("LA_GEN_CACHE", "/tmp/la_gen_cache")
 FIELDS = ("contig_seq", "contig_off", "read_seq", "read_qual", "read_off", "end_read_off")
@@ -89,7 +90,7 @@ def load_workload(config, seed, scale, mmap=False):
     """(batch, params) of a deterministic synthetic workload (a pure function of config, seed,
     scale), cached on local disk; mmap=True maps the cached arrays read-only instead of loading."""
     from gen import Batch, make, seed_for
-    idx = {"C1": 0, "C2": 1, "C3": 2, "C4": 3, "C4S": 3}[config]
+    idx = {"C1": 0, "C2": 1, "C3": 2, "C4": 3, "C4S": 3, "C4F": 3}[config]
     seed = seed_for(idx) + seed
     d = _cache_dir(config, seed, scale)
     if os.path.exists(os.path.join(d, "ok")):
@@ -98,7 +99,7 @@ def load_workload(config, seed, scale, mmap=False):
             return Batch(*arrs), workload_params(config)
         except Exception:
             pass
-    kw = {"scale": scale} if config in ("C2", "C4", "C4S") else {}
+    kw = {"scale": scale} if config in ("C2", "C4", "C4S", "C4F") else {}
     t = time.time()
     b = make(config, seed=seed, **kw)
     log(f"[bench] generated {config} seed {seed}: {b.n_contigs} contigs, {b.n_reads} reads in {time.time() - t:.1f}s")
@@ -358,7 +359,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C4", choices=["C1", "C2", "C3", "C4", "C4S"])
+    ap.add_argument("--config", default="C4", choices=["C1", "C2", "C3", "C4", "C4S", "C4F"])
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],

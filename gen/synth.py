@@ -17,7 +17,7 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-from .batch import Batch, _ranges_to_ids
+from .batch import Batch, _gather_ranges, _ranges_to_ids
 
 ASCII = np.frombuffer(b"ACGTN", np.uint8)
 RL = 150                      # read length (150 bp reads)
@@ -384,6 +384,26 @@ def c4_cfg(seed: int = seed_for(3), scale: float = 1.0, cut_rate: float = 1 / 40
     return MetaCfg("C4", sp)
 
 
+def fig3_subsample(b: Batch, seed: int, zero: float = 0.70, light: float = 0.29) -> Batch:
+    """The paper's bin mix (Fig 3, arcticsynth): "the majority of contigs have zero reads",
+    10-30% have fewer than 10, "less than 1%" the rest.  Applied per contig end to a C4 batch: with
+    probability `zero` the end keeps no reads, with `light` the first U{1..9} of its reads (all if it
+    has fewer), otherwise (1%) all of them (C4's heavy ends: up to ~700 reads; the paper's up to 3000)."""
+    rng = np.random.default_rng(seed ^ 0xF163)
+    r = np.diff(b.end_read_off)
+    u = rng.random(r.shape[0])
+    keep = np.where(u < zero, 0, np.where(u < zero + light, np.minimum(r, rng.integers(1, 10, r.shape[0])), r))
+    read_ids = _ranges_to_ids(b.end_read_off[:-1], keep)
+    rlen = np.diff(b.read_off)[read_ids]
+    roff = np.zeros(read_ids.shape[0] + 1, np.int64)
+    roff[1:] = np.cumsum(rlen)
+    eoff = np.zeros(r.shape[0] + 1, np.int64)
+    eoff[1:] = np.cumsum(keep)
+    rseq = _gather_ranges(b.read_seq, b.read_off[read_ids], rlen)
+    rqual = _gather_ranges(b.read_qual, b.read_off[read_ids], rlen)
+    return Batch(b.contig_seq, b.contig_off, rseq, rqual, roff, eoff, dict(b.meta, fig3_subsample=True))
+
+
 def make(config: str, seed: int | None = None, **kw) -> Batch:
     """Build a named workload: C1, C2, C3, C4 (C5 = C4 sharded, see the multi-GPU driver)."""
     config = config.upper()
@@ -398,6 +418,9 @@ def make(config: str, seed: int | None = None, **kw) -> Batch:
     if config in ("C4", "C5"):
         s = seed if seed is not None else seed_for(3)
         return make_metagenome(c4_cfg(s, kw.pop("scale", 1.0)), s, **kw)
+    if config == "C4F":   # C4 with the paper's Fig 3 mix of reads per end (fig3_subsample)
+        s = seed if seed is not None else seed_for(3)
+        return fig3_subsample(make_metagenome(c4_cfg(s, kw.pop("scale", 1.0)), s, **kw), s)
     if config == "C4S":   # r01's C4 (510k contigs, 31.7M read copies): quicker A/B comparisons
         s = seed if seed is not None else seed_for(3)
         return make_metagenome(c4_cfg(s, kw.pop("scale", 1.0), cut_rate=1 / 2000), s, **kw)
