@@ -58,6 +58,12 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_DEAD0
 #define LA_DEAD0 1   // decide attempts whose start k-mer fails the filter without building (inl32_build_link)
 #endif
+#ifndef LA_WALK_PIPE
+#define LA_WALK_PIPE 1   // software-pipelined walker loop (walk_links)
+#endif
+#ifndef LA_WALK_PIPE_SMALL
+#define LA_WALK_PIPE_SMALL 0   // k_small: thread 0 walks with walk_links (pipelined) instead of its plain loop
+#endif
 #ifndef LA_MAX_LOAD
 #define LA_MAX_LOAD 0.70f
 #endif
@@ -250,8 +256,19 @@ __host__ __device__ __forceinline__ XlcLayout xlc_layout(uint32_t bytes, int r, 
 // Routing estimate of the filtered table: distinct k-mers with >= 2 voting occurrences plus filter
 // false positives, as a fraction of the occurrences (measured on C2/C4 samples: 0.05-0.2, higher for
 // ends with few reads).  A wrong guess only costs a redo in the global path.
+// r02b (LA_FRAC_V2): finer buckets from the measured claims per occurrence (k-mers seen >= 2 times plus
+// the expected filter false positives, 4 bits per occurrence per bitmap) on C4 ends at k = 21 and 33:
+// maxima 0.34 / 0.33 / 0.22 / 0.14 / 0.11 / 0.06 / 0.085 for r < 10 / 25 / 50 / 100 / 200 / 400 / more
+// (DESIGN.md §7); r01's three buckets (0.30 / 0.16 / 0.10) over-reserved the large ends ~1.7x.
+#ifndef LA_FRAC_V2
+#define LA_FRAC_V2 1
+#endif
 __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
+#if LA_FRAC_V2
+    return r < 10 ? 0.36f : (r < 25 ? 0.34f : (r < 50 ? 0.24f : (r < 100 ? 0.16f : (r < 200 ? 0.12f : (r < 400 ? 0.075f : 0.095f)))));
+#else
     return r < 50 ? 0.30f : (r < 200 ? 0.16f : 0.10f);
+#endif
 }
 
 __host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { return 4u * threads; }
@@ -760,6 +777,41 @@ __device__ __forceinline__ int walk_links(uint32_t *info, uint32_t node, int W, 
     int i = 0;
     uint32_t pack = 0;
     term = T_MAXLEN;
+#if LA_WALK_PIPE
+    // software-pipelined: the successor's word is loaded before this step's checks resolve, so the
+    // load latency overlaps the branch; the only word that can change in between is this node's own
+    // (its visited bit), patched in when the successor is the node itself
+    if (W > 0) {
+        if (node == NEXT_NONE) {
+            term = T_DEADEND;
+        } else {
+            uint32_t inf = info[node];
+            for (;;) {
+                const uint32_t nx = inf >> 4, code = inf & 7u;
+                const uint32_t pre = info[nx == NEXT_NONE ? node : nx];   // speculative, always a valid slot
+                if ((inf & 8u) | (code >= 4u)) {   // visited (loop check before the lookup) / fork / dead end
+                    term = (inf & 8u) ? T_LOOP : (code == CODE_FORK ? T_FORK : T_DEADEND);
+                    break;
+                }
+                info[node] = inf | 8u;
+                pack |= ((0x54474341u >> (8 * code)) & 0xffu) << (8 * (i & 3));   // "ACGT"[code]
+                if ((i & 3) == 3) {
+                    *(uint32_t *)(wb + i - 3) = pack;
+                    pack = 0;
+                }
+                ++i;
+                if (i >= W) break;                                    // MAXLEN: no lookup after the W-th base
+                if (nx == NEXT_NONE) {
+                    term = T_DEADEND;
+                    break;
+                }
+                inf = nx == node ? (pre | 8u) : pre;
+                node = nx;
+            }
+        }
+    }
+    if (false)
+#endif
     for (; i < W; ++i) {
         if (node == NEXT_NONE) {
             term = T_DEADEND;
@@ -1598,7 +1650,6 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 B.nclaim = 0;
                 B.dead0 = 0;
                 B.ctr_f = B.ctr_b = 0;
-            B.ctr_f = B.ctr_b = 0;
             }
             const long long tc = la_clock();
             {
@@ -1646,6 +1697,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                 uint32_t node = B.start == NONE ? NEXT_NONE : B.start;
                 int len = 0, term = T_MAXLEN;
                 unsigned long long steps = 0;
+#if LA_WALK_PIPE_SMALL
+                len = walk_links(info, node, P.W, wb, term, steps);
+                if (false)
+#endif
                 for (int i = 0; i < P.W; ++i) {
                     ++steps;   // a lookup; the loop check of a present k-mer precedes it (below)
                     if (node == NEXT_NONE) { term = T_DEADEND; break; }

@@ -10,7 +10,7 @@ for spec in "$@"; do
   i=$((i+1))
   v=${spec%%:*}; envs=""; [[ "$spec" == *:* ]] && envs=${spec#*:}
   tag=$(echo "$spec" | tr -c 'A-Za-z0-9_\n' '_')
-  ( IFS=','; for kv in $envs; do export "$kv"; done
+  ( IFS=','; for kv in $envs; do export "$kv"; done; unset IFS
     LA_SO=$PWD/build_ab/$v.so LA_SERIAL_CLASSES=${SERIAL:-1} timeout ${RUN_TIMEOUT:-300} python bench.py --config ${CFG:-C4S} --steps ${STEPS:-5} --warmup 2 \
       --no-e2e --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/ab_${tag}_${rep}.json 2> gpurun_out/ab_${tag}_${rep}.err )
   python - "$tag" "$rep" <<'PY'

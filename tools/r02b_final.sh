@@ -10,6 +10,7 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/r02b
 timeout 1500 python bench.py --steps 10 --warmup 3 > gpurun_out/r02b_bench_c4.json 2> gpurun_out/r02b_bench_c4.err; echo "c4 rc=$?"
 timeout 900 python bench.py --config C4S --steps 10 --warmup 3 --no-select > gpurun_out/r02b_bench_c4s.json 2> gpurun_out/r02b_bench_c4s.err; echo "c4s rc=$?"
 timeout 900 python bench.py --config C3 --steps 10 --warmup 3 --no-select > gpurun_out/r02b_bench_c3.json 2> gpurun_out/r02b_bench_c3.err; echo "c3 rc=$?"
+timeout 900 python bench.py --config C4F --steps 10 --warmup 3 --no-select > gpurun_out/r02b_bench_c4f.json 2> gpurun_out/r02b_bench_c4f.err; echo "c4f rc=$?"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/r02b_launches_c4.csv \
   python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --no-replay --no-select --coexec-share 0 > /dev/null 2>&1; echo "launches rc=$?"
 timeout 900 bash tools/ncu_traffic.sh r02b_c4s > gpurun_out/r02b_c4s_traffic.txt 2>&1; echo "traffic rc=$?"
