@@ -64,6 +64,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_WALK_PIPE_SMALL
 #define LA_WALK_PIPE_SMALL 0   // k_small: thread 0 walks with walk_links (pipelined) instead of its plain loop
 #endif
+#ifndef LA_STREAM_BIG
+#define LA_STREAM_BIG 1   // largest shared-memory class also takes ends whose reads stay in global memory
+#endif
 #ifndef LA_MAX_LOAD
 #define LA_MAX_LOAD 0.70f
 #endif
@@ -150,10 +153,10 @@ __host__ __device__ __forceinline__ uint32_t cnt_bytes(bool gt, bool wide = fals
 __host__ __device__ __forceinline__ bool xl_wide(uint32_t U) { return U >= 65536u; }
 
 __host__ __device__ __forceinline__ SmemTab smem_tab(const SmemFixed &F, uint32_t U, bool allow_filter,
-                                                     uint32_t kbytes, int r, bool gt, int SW) {
+                                                     uint32_t kbytes, int r, bool gt, int SW, bool staged = true) {
     const bool wide = gt && xl_wide(U);
     SmemTab T;
-    const uint32_t sb = gt ? 0u : stage_bytes(r, SW);   // shared-memory tables: reads staged first
+    const uint32_t sb = (gt || !staged) ? 0u : stage_bytes(r, SW);   // shared-memory tables: reads staged first
     const uint32_t pb = pref_bytes(r) + sb;
     const uint32_t tab = F.tab_bytes > pb ? F.tab_bytes - pb : 0u;
     const uint32_t per_slot = kbytes + cnt_bytes(gt, wide) + 2u;   // key + counters + claim-list entry (u16)
@@ -274,13 +277,13 @@ __host__ __device__ __forceinline__ float filtered_fraction(int64_t r) {
 __host__ __device__ __forceinline__ uint32_t min_table_cap(uint32_t threads) { return 4u * threads; }
 
 __device__ __forceinline__ bool fits(int64_t r, int64_t U, const DevParams &P, uint32_t bytes, uint32_t threads,
-                                     int SW, bool single) {
+                                     int SW, bool single, bool stream = false) {
     const uint32_t min_cap = min_table_cap(threads);
     if (bytes == 0) return false;
     const SmemFixed F = smem_fixed(P.W, bytes, 0u, single, single ? (int)(threads / 32u) : (int)(threads / 32u) - 1);
     if (F.tab_bytes == 0) return false;
     if (r > 16384) return false;
-    const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r, false, SW);
+    const SmemTab T = smem_tab(F, (uint32_t)U, P.V >= 2, key_bytes(P.k_min), (int)r, false, SW, !stream);
     if (T.cap < min_cap) return false;
     if (T.mwords == 0) return true;   // U <= 0.7 cap: cannot overflow
     return filtered_fraction(r) * (float)U + 64.f <= SMEM_MAX_LOAD * (float)T.cap;
@@ -321,8 +324,13 @@ __host__ __device__ __forceinline__ uint32_t xl_stride(int64_t r_max, int64_t U_
 
 // class-list entries: the end id, bit 30 set when a read of the end has an N (list_end / list_anyn)
 constexpr int32_t LIST_ANYN = 1 << 30;
-__host__ __device__ __forceinline__ int list_end(int32_t v) { return v & (LIST_ANYN - 1); }
+// bit 29: the end's reads are read from global memory (L1/L2) instead of being staged in shared memory
+// (largest shared-memory class only, for ends whose staged reads would leave too little room for the
+// table; r02b, LA_STREAM_BIG)
+constexpr int32_t LIST_STREAM = 1 << 29;
+__host__ __device__ __forceinline__ int list_end(int32_t v) { return v & (LIST_STREAM - 1); }
 __host__ __device__ __forceinline__ bool list_anyn(int32_t v) { return (v & LIST_ANYN) != 0; }
+__host__ __device__ __forceinline__ bool list_stream(int32_t v) { return (v & LIST_STREAM) != 0; }
 
 __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restrict__ roff,
                        const uint8_t *__restrict__ rflag,
@@ -352,9 +360,16 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         }
         c = CLS_GLOBAL;
         int sc = -1;
+        bool stream = false;
         if (U < (1ll << 30))
             for (int i = 0; i < N_SMEM_CLASSES && sc < 0; ++i)
                 if (fits(r, U, P, pb.b[i], pb.t[i], SW, (pb.single >> i) & 1u)) sc = i;
+        // the largest class with the reads left in global memory (L1/L2), before the L2-table XL class
+        if (LA_STREAM_BIG && sc < 0 && U < (1ll << 30) && !((pb.single >> (N_SMEM_CLASSES - 1)) & 1u) &&
+            fits(r, U, P, pb.b[N_SMEM_CLASSES - 1], pb.t[N_SMEM_CLASSES - 1], SW, false, true)) {
+            sc = N_SMEM_CLASSES - 1;
+            stream = true;
+        }
         U0 = U0 > 0xffffffffll ? 0xffffffffll : U0;
         // XLC: the table split over a 2-CTA cluster's shared memory (no staging assumed; U < 65536)
         if (sc < 0 && xlc_bytes && P.V >= 2 && r <= 16384 && U <= XLC_MAX_U &&
@@ -369,7 +384,7 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         if (sc >= 0) {
             c = CLS_S + sc;
             const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : (sc == C_XLC ? 11 : sc)], 1);
-            lists[sc * n_ends + i] = (int32_t)e | (anyN ? LIST_ANYN : 0);
+            lists[sc * n_ends + i] = (int32_t)e | (anyN ? LIST_ANYN : 0) | (stream ? LIST_STREAM : 0);
             keys[sc * n_ends + i] = (uint32_t)U0;
             if (sc == N_SMEM_CLASSES) {
                 atomicMax(&ctr[9], (int)U);
@@ -673,6 +688,7 @@ struct EndSlot {            // one contig end in flight
     uint32_t start;         // the start k-mer's slot (NONE if absent) of the last build
     int rec_att;            // replay: attempts recorded by the extension
     int anyN;               // some read of the end has an N (from the class list entry)
+    int stream;             // the end's reads stay in global memory (LIST_STREAM)
     unsigned long long ins, steps;
 };
 
@@ -1306,6 +1322,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                 } else {
                     E.e = e;
                     E.anyN = list_anyn(lv);
+                    E.stream = !GT && list_stream(lv);
                     E.r0 = eoff[e];
                     E.r = (int)(eoff[e + 1] - E.r0);
                     E.ulen = -1;   // unknown until the first prefix pass
@@ -1349,17 +1366,18 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
         // every builder access is a plain LDS (the pointers below are shared-memory pointers whenever
         // !GT, so the compiler emits LDS, not generic loads); the XL class streams them from HBM/L2.
         unsigned char *stage = tbase + FX.off_tab;
-        const bool no_room = !GT && stage_bytes(r, SW) + pref_bytes(r) + 64u * 24u > FX.tab_bytes;
+        const bool stream = !GT && E.stream;   // reads from global memory, like the XL class
+        const bool no_room = !GT && (stream ? 0u : stage_bytes(r, SW)) + pref_bytes(r) + 64u * 24u > FX.tab_bytes;
         uint64_t *sR = (uint64_t *)stage;
         uint64_t *sQ = sR + (size_t)r * SW;
         uint16_t *sL = (uint16_t *)(sQ + (size_t)r * SW);
         uint8_t *sF = (uint8_t *)(sL + r);
-        const uint64_t *gR = GT ? rseq : sR;
-        const uint64_t *gQ = GT ? rqc : sQ;
-        const uint16_t *gL = GT ? rlen : sL;
-        const uint8_t *gF = GT ? rflag : sF;
-        long long lr0 = GT ? r0 : 0;   // first read index in (gR, gQ, gL, gF)
-        if (!GT && !no_room) {
+        const uint64_t *gR = (GT || stream) ? rseq : sR;
+        const uint64_t *gQ = (GT || stream) ? rqc : sQ;
+        const uint16_t *gL = (GT || stream) ? rlen : sL;
+        const uint8_t *gF = (GT || stream) ? rflag : sF;
+        long long lr0 = (GT || stream) ? r0 : 0;   // first read index in (gR, gQ, gL, gF)
+        if (!GT && !stream && !no_room) {
             const uint4 *a4 = (const uint4 *)(rseq + r0 * SW);
             const uint4 *b4 = (const uint4 *)(rqc + r0 * SW);
             const int n4 = r * SW / 2;   // SW is even
@@ -1374,7 +1392,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             builders_sync(NB);
         }
         // positions with a following base, per read (exclusive prefix, pref[r] = U) -> table plan
-        uint32_t *pref = (uint32_t *)(stage + (GT ? 0u : stage_bytes(r, SW)));
+        uint32_t *pref = (uint32_t *)(stage + ((GT || stream) ? 0u : stage_bytes(r, SW)));
         if (no_room) {   // the reads alone do not fit this CTA's shared memory: no table (overflow)
         } else {
             read_prefix(B, E, pref, gL, lr0, r, k, ulen, bt, NB);
@@ -1416,7 +1434,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             }
         }
         if (bt == 0) {   // the attempt's table layout, once (broadcast through shared memory)
-            SmemTab tb = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW);
+            SmemTab tb = smem_tab(FXt, U, P.V >= 2, key_bytes(k), r, GT, SW, !stream);
             if (GT) {   // XL: size the global table for this end (less to clear, scan and cache)
                 const uint32_t need = max(xl_needed_cap(r, U, tb.mwords != 0), min_table_cap(BLOCK));
                 if (tb.cap > need) {
