@@ -33,3 +33,11 @@ def cached_batch(name, **kw):
     if key not in _cache:
         _cache[key] = make(name, **kw)
     return _cache[key]
+
+
+@pytest.fixture(scope="session", autouse=True)
+def _library_up_to_date():
+    """Rebuild liblocassm.so if any CUDA/C++ source is newer than it (no-op when up to date), so the
+    tests never exercise a stale library."""
+    from paper_conf_sc_awanhedbdoy21_b200 import build
+    build.build()
