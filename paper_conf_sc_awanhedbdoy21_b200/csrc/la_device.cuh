@@ -24,6 +24,7 @@ enum : int { T_DEADEND = 0, T_FORK = 1, T_LOOP = 2, T_MAXLEN = 3, T_NOREADS = 4,
 struct DevParams {
     int k_start, k_min, k_max, k_shift, W, qual_offset, q_lo, q_hi, V, F;
     int replay;   // 1: build-only replay of the recorded attempts (la_replay_build); 0: extension
+    int maxlen;   // longest read of the batch (LIST_UNIFORM ends: every read has this length)
 };
 
 __host__ __device__ __forceinline__ int kwords(int k) { return (2 * k + 63) >> 6; }

@@ -64,6 +64,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_WALK_PIPE_SMALL
 #define LA_WALK_PIPE_SMALL 0   // k_small: thread 0 walks with walk_links (pipelined) instead of its plain loop
 #endif
+#ifndef LA_UNIFORM_FLAG
+#define LA_UNIFORM_FLAG 1   // planner marks ends whose reads all have the batch's longest length
+#endif
 #ifndef LA_STREAM_BIG
 #define LA_STREAM_BIG 1   // largest shared-memory class also takes ends whose reads stay in global memory
 #endif
@@ -328,7 +331,12 @@ constexpr int32_t LIST_ANYN = 1 << 30;
 // (largest shared-memory class only, for ends whose staged reads would leave too little room for the
 // table; r02b, LA_STREAM_BIG)
 constexpr int32_t LIST_STREAM = 1 << 29;
-__host__ __device__ __forceinline__ int list_end(int32_t v) { return v & (LIST_STREAM - 1); }
+// bit 28: every read of the end has the batch's longest length (P.maxlen): the first attempt's prefix
+// pass is arithmetic (r02b: the planner already reads every length; the length scan was ~5% of the
+// builders' time)
+constexpr int32_t LIST_UNIFORM = 1 << 28;
+__host__ __device__ __forceinline__ int list_end(int32_t v) { return v & (LIST_UNIFORM - 1); }
+__host__ __device__ __forceinline__ bool list_uniform(int32_t v) { return (v & LIST_UNIFORM) != 0; }
 __host__ __device__ __forceinline__ bool list_anyn(int32_t v) { return (v & LIST_ANYN) != 0; }
 __host__ __device__ __forceinline__ bool list_stream(int32_t v) { return (v & LIST_STREAM) != 0; }
 
@@ -352,11 +360,13 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         // the schedule (table sizing) and at k_start (LPT key); reads shorter than k contribute 0
         int64_t U = 0, U0 = 0;
         int anyN = 0;   // some read of the end has an N: only then do the passes test k-mer windows for N
+        bool uni = true;   // every read has length P.maxlen
         for (int64_t j = eoff[e]; j < eoff[e + 1]; ++j) {
             const int64_t l = roff[j + 1] - roff[j];
             U += l > P.k_min ? l - P.k_min : 0;
             U0 += l > P.k_start ? l - P.k_start : 0;
             anyN |= rflag[j];
+            uni &= l == P.maxlen;
         }
         c = CLS_GLOBAL;
         int sc = -1;
@@ -384,7 +394,8 @@ __global__ void k_plan(const int64_t *__restrict__ eoff, const int64_t *__restri
         if (sc >= 0) {
             c = CLS_S + sc;
             const int i = atomicAdd(&ctr[sc == N_SMEM_CLASSES ? 8 : (sc == C_XLC ? 11 : sc)], 1);
-            lists[sc * n_ends + i] = (int32_t)e | (anyN ? LIST_ANYN : 0) | (stream ? LIST_STREAM : 0);
+            lists[sc * n_ends + i] =
+                (int32_t)e | (anyN ? LIST_ANYN : 0) | (stream ? LIST_STREAM : 0) | (uni && LA_UNIFORM_FLAG ? LIST_UNIFORM : 0);
             keys[sc * n_ends + i] = (uint32_t)U0;
             if (sc == N_SMEM_CLASSES) {
                 atomicMax(&ctr[9], (int)U);
@@ -1325,7 +1336,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                     E.stream = !GT && list_stream(lv);
                     E.r0 = eoff[e];
                     E.r = (int)(eoff[e + 1] - E.r0);
-                    E.ulen = -1;   // unknown until the first prefix pass
+                    E.ulen = list_uniform(lv) ? P.maxlen : -1;   // else unknown until the first prefix pass
                     E.kmax_eff = min(P.k_max, (int)clen[e]);
                     E.k = P.k_start;
                     E.shift = 0;
@@ -1584,7 +1595,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
                     E.anyN = list_anyn(lv);
                 E.r0 = eoff[e];
                 E.r = (int)(eoff[e + 1] - E.r0);
-                E.ulen = -1;
+                E.ulen = list_uniform(lv) ? P.maxlen : -1;
                 E.kmax_eff = min(P.k_max, (int)clen[e]);
                 E.k = P.k_start;
                 E.shift = 0;

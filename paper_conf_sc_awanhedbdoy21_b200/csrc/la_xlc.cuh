@@ -361,7 +361,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(XLC_THREADS, 1) k_xl
                 E.anyN = list_anyn(lv);
                 E.r0 = eoff[e];
                 E.r = (int)(eoff[e + 1] - E.r0);
-                E.ulen = -1;
+                E.ulen = list_uniform(lv) ? P.maxlen : -1;
                 E.kmax_eff = min(P.k_max, (int)clen[e]);
                 E.k = P.k_start;
                 E.shift = 0;

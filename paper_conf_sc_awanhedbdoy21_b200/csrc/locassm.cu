@@ -534,7 +534,8 @@ extern "C" la_status la_load_batch(la_ctx *ctx, const la_batch *b, const la_para
         CK(grow(E.tailN, std::max<int64_t>(nE, 1) * 16));
         CK(grow(E.clen, std::max<int64_t>(nE, 1) * 4));
         DevParams dp{params->k_start, params->k_min, params->k_max, params->k_shift, params->max_walk_len,
-                     params->qual_offset, params->q_lo, params->q_hi, params->min_votes, params->min_frac_pct, 0};
+                     params->qual_offset, params->q_lo, params->q_hi, params->min_votes, params->min_frac_pct, 0,
+                     maxlen};
         if (nR) {
             CK(cudaMemsetAsync(E.rflag.p, 0, nR, st));
             k_read_end<<<blocks(nR, 256), 256, 0, st>>>(P<int64_t>(E.eoff), nE, nR, P<int32_t>(ctx->read_end));

@@ -1,7 +1,7 @@
 #!/bin/bash
 # A/B of library variants (built HERE by tools/ab_build.sh into build_ab/<name>.so): serial-class C4S
 # bench per variant on the same GPU box, kernel path only.
-#   gpurun -- bash tools/ab.sh name1 "name2:ENV=1,ENV2=x" ...
+#   gpurun -- bash tools/ab.sh name1 "name2:ENV=1;ENV2=x" ...   (env assignments separated by ';')
 mkdir -p gpurun_out
 timeout 400 python bench.py --config ${CFG:-C4S} --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-replay --no-select --coexec-share 0 > /dev/null 2>&1
 i=0
@@ -10,7 +10,7 @@ for spec in "$@"; do
   i=$((i+1))
   v=${spec%%:*}; envs=""; [[ "$spec" == *:* ]] && envs=${spec#*:}
   tag=$(echo "$spec" | tr -c 'A-Za-z0-9_\n' '_')
-  ( IFS=','; for kv in $envs; do export "$kv"; done; unset IFS
+  ( IFS=';'; for kv in $envs; do export "$kv"; done; unset IFS
     LA_SO=$PWD/build_ab/$v.so LA_SERIAL_CLASSES=${SERIAL:-1} timeout ${RUN_TIMEOUT:-300} python bench.py --config ${CFG:-C4S} --steps ${STEPS:-5} --warmup 2 \
       --no-e2e --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/ab_${tag}_${rep}.json 2> gpurun_out/ab_${tag}_${rep}.err )
   python - "$tag" "$rep" <<'PY'
