@@ -1,5 +1,5 @@
 /* abi_client.c — a plain C client of include/locassm.h (no Python, no C++): builds a tiny batch,
- * runs la_create -> la_load_batch -> la_extend -> la_get_stats -> la_destroy on cuda:0 and checks
+ * runs la_create -> la_load_batch -> la_extend -> la_get_stats -> la_select_reads -> la_destroy on cuda:0 and checks
  * the result against the closed form of SURVEY.md §8(c) pin P2 (error-free tiled reads, Alg 1/2 of
  * P:L404-448): with reads starting at every a in [a_lo, a_hi] (length l, all Q40), the right walk
  * from contig end e is G[e : a_hi + l - V + 1] with code DEADEND; an end without reads is NOREADS
@@ -31,6 +31,20 @@ static int unique_kmers(const char *g, int n, int k) {
     return 1;
 }
 
+static char comp(char c) { return c == 'A' ? 'T' : (c == 'C' ? 'G' : (c == 'G' ? 'C' : 'A')); }
+
+/* every k-mer of g occurs once counting both strands (N4's closed form needs unique seeds) */
+static int unique_kmers_both(const char *g, int n, int k) {
+    char *r = (char *)malloc((size_t)n);
+    for (int i = 0; i < n; ++i) r[i] = comp(g[n - 1 - i]);
+    int ok = unique_kmers(g, n, k);
+    for (int i = 0; ok && i + k <= n; ++i)
+        for (int j = 0; j + k <= n; ++j)
+            if (memcmp(g + i, r + j, (size_t)k) == 0) { ok = 0; break; }
+    free(r);
+    return ok;
+}
+
 #define CHECK(cond, ...)                                            \
     do {                                                            \
         if (!(cond)) {                                              \
@@ -45,7 +59,7 @@ int main(void) {
     do {
         for (int i = 0; i < GLEN; ++i) g[i] = "ACGT"[rnd() & 3u];
         g[GLEN] = 0;
-    } while (!unique_kmers(g, GLEN, 21));
+    } while (!unique_kmers(g, GLEN, 21) || !unique_kmers_both(g, GLEN, 16));
     /* one contig G[300:500); its right end e = 500 has reads starting at a = 200..600 (a_hi = 600),
        its left end has none */
     const int cs = 300, e = 500, a_lo = 200, a_hi = 600, V = 2;
@@ -99,6 +113,61 @@ int main(void) {
     /* results are library-owned: read them before la_destroy */
     printf("abi_client ok: right extension %lld bases (closed form %d), DEADEND, k %d, %d attempts\n",
            (long long)got_len, want_len, r.k_used[1], r.n_attempts[1]);
+
+    /* NEXT N4 (la_select_reads, readings S1-S6): FR pairs from fragments [a, a+350), a = a_lo..a_hi,
+       mate 0 = G[a, a+150), mate 1 = rc(G[a+200, a+350)).  With unique 16-mers on both strands the
+       selection has a closed form: the RIGHT end (window G[350, 500)) takes every pair whose forward
+       read overlaps the window by >= 20 (a in [220, 480]) or whose reverse read does and reaches past
+       500 (a in [200, 280]): a in [200, 480], 281 pairs; the LEFT end (window G[300, 450)) takes the
+       pairs whose reverse read overlaps it by >= 20 (a <= 230) or whose forward read does and starts
+       before 300 (a in [200, 299]): 100 pairs.  The selected batch, loaded on the device and extended,
+       tiles starts 200..680 (forward reads and mates): the right walk passes W = 300 bases (P2 closed
+       form 680 + 150 - V + 1 - 500 = 329 > W): MAXLEN with G[500, 800). */
+    CHECK(unique_kmers_both(g, GLEN, 16), "the genome repeats a 16-mer (on either strand)");
+    {
+        const int np = a_hi - a_lo + 1;
+        char *ps = (char *)malloc((size_t)np * 2 * RLEN), *pq = (char *)malloc((size_t)np * 2 * RLEN);
+        int64_t *po = (int64_t *)malloc(sizeof(int64_t) * (size_t)(2 * np + 1));
+        for (int i = 0; i < np; ++i) {
+            const int a = a_lo + i;
+            memcpy(ps + (size_t)(2 * i) * RLEN, g + a, RLEN);
+            for (int j = 0; j < RLEN; ++j) ps[(size_t)(2 * i + 1) * RLEN + j] = comp(g[a + 349 - j]);
+        }
+        memset(pq, 'I', (size_t)np * 2 * RLEN);
+        for (int i = 0; i <= 2 * np; ++i) po[i] = (int64_t)i * RLEN;
+        la_pool pool;
+        memset(&pool, 0, sizeof pool);
+        pool.mem = LA_MEM_HOST;
+        pool.n_contigs = 1;
+        pool.contig_seq = g + cs;
+        pool.contig_off = coff;
+        pool.n_pairs = np;
+        pool.read_seq = ps;
+        pool.read_qual = pq;
+        pool.read_off = po;
+        la_sel_params sp = {150, 16, 4, 20, 4};
+        la_selection sel;
+        if ((s = la_select_reads(ctx, &pool, &sp, &sel)) != LA_OK) {
+            fprintf(stderr, "abi_client: la_select_reads %d: %s\n", (int)s, la_last_error(ctx));
+            la_destroy(ctx);
+            return 2;
+        }
+        CHECK(sel.n_sel == 281 + 100, "selected (end, pair) records %lld, closed form 381", (long long)sel.n_sel);
+        CHECK(sel.batch.mem == LA_MEM_DEVICE && sel.batch.n_reads == 2 * sel.n_sel, "selection batch");
+        if ((s = la_load_batch(ctx, &sel.batch, &p)) != LA_OK || (s = la_extend(ctx, &r)) != LA_OK) {
+            fprintf(stderr, "abi_client: select -> extend %d: %s\n", (int)s, la_last_error(ctx));
+            la_destroy(ctx);
+            return 2;
+        }
+        CHECK(r.ext_off[2] - r.ext_off[1] == 300 && r.term[1] == LA_TERM_MAXLEN, "selected right end: %lld bases, term %d",
+              (long long)(r.ext_off[2] - r.ext_off[1]), r.term[1]);
+        CHECK(memcmp(r.ext_seq + r.ext_off[1], g + e, 300) == 0, "selected right end != genome continuation");
+        printf("abi_client ok: la_select_reads %lld pairs (closed form 381); extended right end MAXLEN, 300 bases\n",
+               (long long)sel.n_sel);
+        free(ps);
+        free(pq);
+        free(po);
+    }
     CHECK(la_destroy(ctx) == LA_OK, "la_destroy");
     free(rseq);
     free(rqual);
