@@ -353,7 +353,8 @@ def test_replay_build_reruns_the_attempts(LA, orc):
 
 
 def test_c_abi_client():
-    """The plain C client (examples/abi_client.c) on the device: closed-form pin P2 through the ABI."""
+    """The plain C client (examples/abi_client.c) on the device: closed-form pin P2 through the ABI, and
+    the N4 selection's closed-form count followed by the extension of the selected device batch."""
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -363,7 +364,7 @@ def test_c_abi_client():
     exe = os.path.join(root, "examples", "abi_client")
     out = subprocess.run([exe], capture_output=True, text=True, timeout=120)
     assert out.returncode == 0, out.stderr
-    assert "abi_client ok" in out.stdout
+    assert out.stdout.count("abi_client ok") == 2, out.stdout
 
 
 def test_xl_wide_counters(LA, orc):
