@@ -71,7 +71,7 @@ __device__ __forceinline__ long long la_clock() {
 #define LA_STREAM_BIG 1   // largest shared-memory class also takes ends whose reads stay in global memory
 #endif
 #ifndef LA_MAX_LOAD
-#define LA_MAX_LOAD 0.70f
+#define LA_MAX_LOAD 0.80f
 #endif
 constexpr float SMEM_MAX_LOAD = LA_MAX_LOAD;   // table load above which an end overflows (claims)
 
