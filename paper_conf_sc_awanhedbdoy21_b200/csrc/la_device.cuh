@@ -147,6 +147,36 @@ __device__ __forceinline__ int ext_rule(const uint32_t lo[4], const uint32_t hi[
     return m == 0 ? CODE_DEADEND : ((m & (m - 1)) ? CODE_FORK : one);
 }
 
+// Same rule in 32-bit arithmetic, for tables whose counters are bounded well below 2^32 / 100 (the
+// shared-memory classes' 8-bit fields, the XL class's fields for at most XL_MAX_U = 2^21 occurrences):
+// 100 x count and F x total then fit in 32 bits, exactly as the 64-bit products above.
+__device__ __forceinline__ int ext_rule32(const uint32_t lo[4], const uint32_t hi[4], int V, int F) {
+    const uint32_t H = hi[0] + hi[1] + hi[2] + hi[3];
+    const uint32_t L = lo[0] + lo[1] + lo[2] + lo[3];
+    uint32_t mh = 0, ml = 0;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+        mh |= (hi[b] >= (uint32_t)V && 100u * hi[b] >= (uint32_t)F * H) ? (1u << b) : 0u;
+        ml |= (lo[b] >= (uint32_t)V && 100u * lo[b] >= (uint32_t)F * L) ? (1u << b) : 0u;
+    }
+    const uint32_t m = mh ? mh : ml;   // the high tier decides when it has a candidate
+    const int one = __ffs(m) - 1;
+    return m == 0 ? CODE_DEADEND : ((m & (m - 1)) ? CODE_FORK : one);
+}
+
+// N in bases [lo, hi) of a contig tail whose N mask is the 128-bit pair (n0, n1) (bit i = base i):
+// two masked ANDs instead of a per-base loop (reading #5, the start k-mer's N test)
+__device__ __forceinline__ bool any_n_range(uint64_t n0, uint64_t n1, int lo, int hi) {
+    auto rng = [](int a, int b) -> uint64_t {   // bits [a, b) of one 64-bit word, a and b clamped to [0, 64]
+        a = a < 0 ? 0 : (a > 64 ? 64 : a);
+        b = b < 0 ? 0 : (b > 64 ? 64 : b);
+        if (a >= b) return 0ull;
+        const uint64_t upto = b >= 64 ? ~0ull : ((1ull << b) - 1ull);
+        return upto & ~((1ull << a) - 1ull);
+    };
+    return ((n0 & rng(lo, hi)) | (n1 & rng(lo - 64, hi - 64))) != 0ull;
+}
+
 // The k up/down-shift rule (readings #8, #10).  Returns true when the end is done,
 // else updates k / shift for the next attempt.
 __device__ __forceinline__ bool next_k(int term, int &k, int &shift, int kmax_eff, const DevParams &P) {

@@ -64,6 +64,12 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_WALK_PIPE_SMALL
 #define LA_WALK_PIPE_SMALL 0   // k_small: thread 0 walks with walk_links (pipelined) instead of its plain loop
 #endif
+#ifndef LA_NW_ALL4
+#define LA_NW_ALL4 0   // every inline key (k <= 63) on the 4-word path (one code copy)
+#endif
+#ifndef LA_NW_MERGE23
+#define LA_NW_MERGE23 0   // k <= 32 on the 3-word inline path too (one code copy fewer: instruction-cache pressure)
+#endif
 #ifndef LA_UNIFORM_FLAG
 #define LA_UNIFORM_FLAG 1   // planner marks ends whose reads all have the batch's longest length
 #endif
@@ -895,7 +901,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     if (bt == 0) {
         const int p = Tn - k;
         bool hasN = false;
-        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
+        hasN = any_n_range(n0, n1, p, Tn);
         uint32_t Tw[2 * TAIL_W];
 #pragma unroll
         for (int i = 0; i < TAIL_W; ++i) {
@@ -1051,7 +1057,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
             K = key_of<NW>(ld_slot<GT>(T, s));
             uint32_t lo[4], hi[4];
             votes32<GT>(T, s, lo, hi);
-            code = ext_rule(lo, hi, P.V, P.F);
+            code = ext_rule32(lo, hi, P.V, P.F);
             if (code < 4) roll32<NW>(K, k, (uint32_t)code);
         }
         const uint32_t h = hash32<NW>(K);
@@ -1070,8 +1076,8 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                            long long &t_filter, long long &t_build, bool replay, int ulen, void *fpos,
                                            uint32_t *queue, bool anyN) {
     if (INL) {
-        const int nw = kw32(T.k);
-        if (nw <= 2)
+        const int nw = LA_NW_ALL4 ? 4 : kw32(T.k);
+        if (nw <= 2 && !LA_NW_MERGE23)
             inl32_build_link<2, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else if (nw == 3)
@@ -1130,7 +1136,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                 K = extract_kmer<MAX_KW>(T.rseq + (size_t)slot_read(w) * T.SW, slot_pos(w), k, KW);
                 uint32_t lo[4], hi[4];
                 votes_of<GT>(T, s, lo, hi);
-                code = ext_rule(lo, hi, P.V, P.F);
+                code = ext_rule32(lo, hi, P.V, P.F);
                 if (code < 4) roll_kmer(K, k, KW, (uint32_t)code);
             }
             const uint32_t t = warp_lookup_ref<GT>(T, has && code < 4, K, hash_kmer(K, KW));
@@ -1141,7 +1147,7 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
         // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
         const int p = Tn - k;
         bool hasN = false;
-        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
+        hasN = any_n_range(n0, n1, p, Tn);
         uint32_t st = NONE;
         if (!hasN) {
             uint64_t Tw[TAIL_W];

@@ -237,7 +237,7 @@ __device__ __forceinline__ void xlc_passes(BuildCtl &B, const TabC &T, uint32_t 
     if (tid == 0) {   // start k-mer: last k bases of the oriented contig (Alg 2 line 4; reading #6)
         const int p = Tn - k;
         bool hasN = false;
-        for (int i = p; i < Tn; ++i) hasN |= ((i < 64 ? n0 >> i : n1 >> (i - 64)) & 1ull) != 0;
+        hasN = any_n_range(n0, n1, p, Tn);
         uint32_t Tw[2 * TAIL_W];
 #pragma unroll
         for (int i = 0; i < TAIL_W; ++i) {
