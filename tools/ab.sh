@@ -12,7 +12,7 @@ for spec in "$@"; do
   tag=$(echo "$spec" | tr -c 'A-Za-z0-9_\n' '_')
   ( IFS=';'; for kv in $envs; do export "$kv"; done; unset IFS
     LA_SO=$PWD/build_ab/$v.so LA_SERIAL_CLASSES=${SERIAL:-1} timeout ${RUN_TIMEOUT:-300} python bench.py --config ${CFG:-C4S} --steps ${STEPS:-5} --warmup 2 \
-      --no-e2e --no-cpu-baseline ${BENCH_ARGS:-} > gpurun_out/ab_${tag}_${rep}.json 2> gpurun_out/ab_${tag}_${rep}.err )
+      --no-e2e ${PARITY_ARGS:---no-cpu-baseline} ${BENCH_ARGS:-} > gpurun_out/ab_${tag}_${rep}.json 2> gpurun_out/ab_${tag}_${rep}.err )
   python - "$tag" "$rep" <<'PY'
 import json, sys
 v, rep = sys.argv[1], sys.argv[2]
@@ -22,7 +22,8 @@ except Exception as e:
     print(v, rep, "FAILED", e); sys.exit(0)
 w = d["work"]["classes"]
 rb = d.get("roofline_build") or {}
-print(f"{v:28s} r{rep} ms/step {d['ms_per_step']:7.2f} build {rb.get('ms') or 0:7.2f} xl {d['work']['ends_xl']} ovf {d['work']['ends_by_class'][4]} "
+par = d.get("parity") or {}
+print(f"{v:28s} r{rep} parity {par.get('mismatches', '-')}/{par.get('ends_checked', '-')} ms/step {d['ms_per_step']:7.2f} build {rb.get('ms') or 0:7.2f} xl {d['work']['ends_xl']} ovf {d['work']['ends_by_class'][4]} "
       + " ".join(f"{c['ends']//1000}k:{c['ms']:.1f}/{c['inserts']/max(c['ms'],1e-9)/1e6:.0f}G" for k, c in w.items()))
 PY
 done; done
