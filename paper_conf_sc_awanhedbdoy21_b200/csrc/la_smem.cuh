@@ -64,11 +64,8 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_WALK_PIPE_SMALL
 #define LA_WALK_PIPE_SMALL 0   // k_small: thread 0 walks with walk_links (pipelined) instead of its plain loop
 #endif
-#ifndef LA_NW_ALL4
-#define LA_NW_ALL4 0   // every inline key (k <= 63) on the 4-word path (one code copy)
-#endif
 #ifndef LA_NW_MERGE23
-#define LA_NW_MERGE23 0   // k <= 32 on the 3-word inline path too (one code copy fewer: instruction-cache pressure)
+#define LA_NW_MERGE23 1   // k <= 32 on the 3-word inline path too (one code copy fewer: instruction-cache pressure)
 #endif
 #ifndef LA_UNIFORM_FLAG
 #define LA_UNIFORM_FLAG 1   // planner marks ends whose reads all have the batch's longest length
@@ -1067,6 +1064,9 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
     if (bt == 0) B.start = B.start_ok ? lookup32<GT>(T, key_form<NW>(Kst, B.start_h), B.start_h) : NONE;
 }
 
+// Each inline-key width NW is a full copy of the filter / build / link passes, and the table kernels
+// are sensitive to instruction-cache pressure (r02b: C4 attempts run k = 33 then 25, which were two
+// hot copies, NW = 3 and 2); LA_NW_MERGE23 runs both on the 3-word code.
 template <bool INL, bool GT>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
@@ -1076,11 +1076,13 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                            long long &t_filter, long long &t_build, bool replay, int ulen, void *fpos,
                                            uint32_t *queue, bool anyN) {
     if (INL) {
-        const int nw = LA_NW_ALL4 ? 4 : kw32(T.k);
-        if (nw <= 2 && !LA_NW_MERGE23)
+        // LA_NW_MERGE23: 17 <= k <= 32 on the 3-word code (the masks of kmask32 cover the last two words,
+        // so a 3-word k-mer needs k >= 17); k <= 16 keeps the 2-word code
+        const int nw = kw32(T.k);
+        if (nw <= 2 && !(LA_NW_MERGE23 && T.k >= 17))
             inl32_build_link<2, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
-        else if (nw == 3)
+        else if (nw <= 3)
             inl32_build_link<3, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else
