@@ -45,6 +45,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_FQUEUE
 #define LA_FQUEUE 0   // 1: filtered builds keep per-position filter indices and queue survivors (r02 experiment)
 #endif
+#ifndef LA_SMALL_FILTER_UNROLL
+#define LA_SMALL_FILTER_UNROLL 2   // the same in k_small (less code per copy with 1: instruction-cache pressure)
+#endif
 #ifndef LA_FILTER_UNROLL
 #define LA_FILTER_UNROLL 2   // positions per lane per iteration of the filter pass (la_inl32.cuh)
 #endif
@@ -873,7 +876,7 @@ __device__ __forceinline__ uint32_t link_info(int code, uint32_t nxt) {
 
 // Inline keys (k <= 63) on 32-bit words (la_inl32.cuh): filter pass, build pass (Alg 1), link pass
 // (a5) and the start k-mer's slot, for NW = ceil(2k/32) words.
-template <int NW, bool GT>
+template <int NW, bool GT, int UF = LA_FILTER_UNROLL>
 __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, uint32_t *B1, uint32_t *B2,
                                                  uint32_t mbits, uint32_t *info, const uint64_t *__restrict__ rqc,
                                                  const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
@@ -935,10 +938,10 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                      }
                                  };
             if (LA_DYN && !GT && ulen > k)
-                warp_positions32_dyn<NW, LA_FILTER_UNROLL>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
+                warp_positions32_dyn<NW, UF>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
                                                            &B.ctr_f, filt);
             else
-                warp_positions32<NW, LA_FILTER_UNROLL>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
+                warp_positions32<NW, UF>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
                                                        stop, filt);
             builders_sync(NB);
             // The filter has no false negatives: a start k-mer whose B2 bit is clear has < 2 voting
@@ -1067,7 +1070,7 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
 // Each inline-key width NW is a full copy of the filter / build / link passes, and the table kernels
 // are sensitive to instruction-cache pressure (r02b: C4 attempts run k = 33 then 25, which were two
 // hot copies, NW = 3 and 2); LA_NW_MERGE23 runs both on the 3-word code.
-template <bool INL, bool GT>
+template <bool INL, bool GT, int UF = LA_FILTER_UNROLL>
 __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_t *B1, uint32_t *B2, uint32_t mbits,
                                            uint32_t *info, const uint64_t *__restrict__ rqc,
                                            const uint16_t *__restrict__ rlen, const uint8_t *__restrict__ rflag,
@@ -1080,13 +1083,13 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
         // so a 3-word k-mer needs k >= 17); k <= 16 keeps the 2-word code
         const int nw = kw32(T.k);
         if (nw <= 2 && !(LA_NW_MERGE23 && T.k >= 17))
-            inl32_build_link<2, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+            inl32_build_link<2, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else if (nw <= 3)
-            inl32_build_link<3, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+            inl32_build_link<3, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         else
-            inl32_build_link<4, GT>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
+            inl32_build_link<4, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
                                     bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
         return;
     }
@@ -1703,7 +1706,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             void *fpos = (void *)(sm + TB.off_f);
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (inline_keys(k))
-                build_link<true, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
+                build_link<true, false, LA_SMALL_FILTER_UNROLL>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
             else
                 build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
