@@ -45,6 +45,9 @@ __device__ __forceinline__ long long la_clock() {
 #ifndef LA_FQUEUE
 #define LA_FQUEUE 0   // 1: filtered builds keep per-position filter indices and queue survivors (r02 experiment)
 #endif
+#ifndef LA_LDS_READS
+#define LA_LDS_READS 1   // staged reads read through 32-bit shared addresses (LDS) in the dyn traversal
+#endif
 #ifndef LA_SMALL_FILTER_UNROLL
 #define LA_SMALL_FILTER_UNROLL 2   // the same in k_small (less code per copy with 1: instruction-cache pressure)
 #endif
@@ -882,7 +885,8 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                                  const uint8_t *__restrict__ rflag, const uint32_t *pref, long long r0,
                                                  int r, int ulen, const DevParams &P, const uint64_t *tail_e, int Tn,
                                                  uint64_t n0, uint64_t n1, int bt, int NB, long long &t_filter,
-                                                 long long &t_build, bool replay, void *fpos, uint32_t *queue, bool anyN) {
+                                                 long long &t_build, bool replay, void *fpos, uint32_t *queue, bool anyN,
+                                                 bool sreads) {
     const volatile int *stop = &B.overflow;
     const int k = TC.k;
     const int lane = bt & 31, wid = bt >> 5, nwarps = NB >> 5;
@@ -937,7 +941,10 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                          }
                                      }
                                  };
-            if (LA_DYN && !GT && ulen > k)
+            if (LA_DYN && !GT && ulen > k && sreads && LA_LDS_READS)
+                warp_positions32_dyn<NW, UF, true>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane,
+                                                   stop, &B.ctr_f, filt);
+            else if (LA_DYN && !GT && ulen > k)
                 warp_positions32_dyn<NW, UF>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
                                                            &B.ctr_f, filt);
             else
@@ -972,7 +979,10 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
             }
             warp_insert32<GT>(T, want, key_form<NW>(K, h), h, nb, hi, lane, &B.nclaim, claim_limit, &B.overflow, pend);
         };
-        if (LA_DYN && !GT && ulen > k)
+        if (LA_DYN && !GT && ulen > k && sreads && LA_LDS_READS)
+            warp_positions32_dyn<NW, 1, true>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
+                                              &B.ctr_b, build);
+        else if (LA_DYN && !GT && ulen > k)
             warp_positions32_dyn<NW, 1>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop, &B.ctr_b, build);
         else
             warp_positions32<NW>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop, build);
@@ -1077,20 +1087,20 @@ __device__ __forceinline__ void build_link(BuildCtl &B, const TabCtx &T, uint32_
                                            const uint32_t *pref, long long r0, int r, const DevParams &P,
                                            const uint64_t *tail_e, int Tn, uint64_t n0, uint64_t n1, int bt, int NB,
                                            long long &t_filter, long long &t_build, bool replay, int ulen, void *fpos,
-                                           uint32_t *queue, bool anyN) {
+                                           uint32_t *queue, bool anyN, bool sreads = false) {
     if (INL) {
         // LA_NW_MERGE23: 17 <= k <= 32 on the 3-word code (the masks of kmask32 cover the last two words,
         // so a 3-word k-mer needs k >= 17); k <= 16 keeps the 2-word code
         const int nw = kw32(T.k);
         if (nw <= 2 && !(LA_NW_MERGE23 && T.k >= 17))
             inl32_build_link<2, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN, sreads);
         else if (nw <= 3)
             inl32_build_link<3, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN, sreads);
         else
             inl32_build_link<4, GT, UF>(B, T, B1, B2, mbits, info, rqc, rflag, pref, r0, r, ulen, P, tail_e, Tn, n0, n1,
-                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN);
+                                    bt, NB, t_filter, t_build, replay, fpos, queue, anyN, sreads);
         return;
     }
     // ---- pointer keys (k >= 64): the same passes with 4-word k-mers ----
@@ -1511,10 +1521,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (INL)
                 build_link<true, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
+                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, !GT && !stream);
             else
                 build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
+                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, !GT && !stream);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
             if (bt == 0) s_acc[6] += B.dead0;
         }
@@ -1707,10 +1717,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_small(
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (inline_keys(k))
                 build_link<true, false, LA_SMALL_FILTER_UNROLL>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                        NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
+                                        NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, true);
             else
                 build_link<false, false>(B, T, B1, B2, mbits, info, sQ, sL, sF, pref, 0, r, P, tail_e, Tn, n0, n1, bt,
-                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0);
+                                         NB, t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, true);
             __syncthreads();
             const long long te = la_clock();
             b_t[1] += tc - tb;
