@@ -404,7 +404,32 @@ __device__ __forceinline__ uint32_t nmask32(uint32_t q) { return q & (q >> 1) & 
 // f(inr, act, g, K, h, nb, hi): inr = this lane has a position g this iteration; act = it is a voting
 // occurrence (q >= q_lo, no N in the window and in the following base).  rflag = nullptr: no read of
 // the end has an N (the class list entry says so), so the k-mer windows are not tested for N.
-template <int NW, int UNR = 1, typename F>
+// SM = true: rseq / rqc are the end's reads staged in shared memory; the word loads then go through
+// 32-bit shared-window addresses (LDS) — through the generic pointers nvcc emitted LD.E with 64-bit
+// address arithmetic (r02b ncu of k_smem<256>: the extraction loads' line was 14% of the instructions)
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+template <int NW>
+__device__ __forceinline__ K32<NW> extract32s(uint32_t rowb, int p, const KMask &m) {
+    const int q = p >> 4, s = (p & 15) << 1;
+    uint32_t x[NW + 1];
+#pragma unroll
+    for (int i = 0; i <= NW; ++i) x[i] = lds32(rowb + 4u * (uint32_t)((q + i) ^ 1));
+    K32<NW> K;
+#pragma unroll
+    for (int i = 0; i < NW; ++i) K.w[i] = __funnelshift_l(x[i + 1], x[i], s);
+    if (NW >= 2) K.w[NW - 2] &= m.m2;
+    K.w[NW - 1] &= m.m1;
+    return K;
+}
+__device__ __forceinline__ uint32_t base32s(uint32_t rowb, int i) {
+    return (lds32(rowb + 4u * (uint32_t)((i >> 4) ^ 1)) >> (30 - ((i & 15) << 1))) & 3u;
+}
+
+template <int NW, int UNR = 1, bool SM = false, typename F>
 __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rseq, const uint32_t *__restrict__ rqc,
                                                  const uint8_t *__restrict__ rflag, const uint32_t *pref,
                                                  long long r0, int r, int SW2, int k, int ulen, int wid, int nwarps,
@@ -414,6 +439,8 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
     const uint32_t we = (uint32_t)(((uint64_t)total * (uint32_t)(wid + 1)) / (uint32_t)nwarps);
     if (wb >= we) return;
     const KMask m = kmask32<NW>(k);
+    const uint32_t sR = SM ? (uint32_t)__cvta_generic_to_shared(rseq) : 0u;   // staged reads (r0 == 0)
+    const uint32_t sQ = SM ? (uint32_t)__cvta_generic_to_shared(rqc) : 0u;
     const uint32_t np = ulen > k ? (uint32_t)(ulen - k) : 1u;
     const uint32_t magic = 0xFFFFFFFFu / np;
     uint32_t g = wb + lane;
@@ -444,8 +471,18 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
                 const int p = act ? (int)pp : 0;
                 const long long row = (r0 + (act ? (int)jj : 0)) * (long long)SW2;
                 const uint32_t *R = rseq + row, *Q = rqc + row;
-                const K32<NW> K = extract32<NW>(R, p, m);
-                const uint32_t nb = base32(R, p + k), nq = base32(Q, p + k);
+                K32<NW> K;
+                uint32_t nb, nq;
+                if (SM) {
+                    const uint32_t rowo = 4u * (uint32_t)row;
+                    K = extract32s<NW>(sR + rowo, p, m);
+                    nb = base32s(sR + rowo, p + k);
+                    nq = base32s(sQ + rowo, p + k);
+                } else {
+                    K = extract32<NW>(R, p, m);
+                    nb = base32(R, p + k);
+                    nq = base32(Q, p + k);
+                }
                 bool vote = act && (nq - 1u < 2u);
                 if (vote && rflag && rflag[r0 + jj]) {
                     const int q = p >> 4, s = (p & 15) << 1;
@@ -483,10 +520,19 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
         }
         const long long row = (r0 + (act ? j : 0)) * (long long)SW2;
         const uint32_t *R = rseq + row, *Q = rqc + row;
-        const K32<NW> K = extract32<NW>(R, act ? p : 0, m);
         const int i = p + k;
-        const uint32_t nb = base32(R, act ? i : 0);
-        const uint32_t nq = base32(Q, act ? i : 0);
+        K32<NW> K;
+        uint32_t nb, nq;
+        if (SM) {
+            const uint32_t rowo = 4u * (uint32_t)row;
+            K = extract32s<NW>(sR + rowo, act ? p : 0, m);
+            nb = base32s(sR + rowo, act ? i : 0);
+            nq = base32s(sQ + rowo, act ? i : 0);
+        } else {
+            K = extract32<NW>(R, act ? p : 0, m);
+            nb = base32(R, act ? i : 0);
+            nq = base32(Q, act ? i : 0);
+        }
         bool vote = act && (nq - 1u < 2u);
         if (vote && rflag && rflag[r0 + j]) {   // reading #5: a k-mer with an N has no entry (rare)
             const int q = p >> 4, s = (p & 15) << 1;
@@ -505,31 +551,6 @@ __device__ __forceinline__ void warp_positions32(const uint32_t *__restrict__ rs
 // Dynamic version for ends whose reads all have length ulen > 0: warps take chunks of 32 * UNR
 // consecutive positions from a shared counter (one atomic per chunk) instead of a fixed 1/nwarps
 // range, so no warp waits at the pass's closing barrier for a slower one (probe rounds differ).
-// SM = true: rseq / rqc are the end's reads staged in shared memory; the word loads then go through
-// 32-bit shared-window addresses (LDS) — through the generic pointers nvcc emitted LD.E with 64-bit
-// address arithmetic (r02b ncu of k_smem<256>: the extraction loads' line was 14% of the instructions)
-__device__ __forceinline__ uint32_t lds32(uint32_t a) {
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-template <int NW>
-__device__ __forceinline__ K32<NW> extract32s(uint32_t rowb, int p, const KMask &m) {
-    const int q = p >> 4, s = (p & 15) << 1;
-    uint32_t x[NW + 1];
-#pragma unroll
-    for (int i = 0; i <= NW; ++i) x[i] = lds32(rowb + 4u * (uint32_t)((q + i) ^ 1));
-    K32<NW> K;
-#pragma unroll
-    for (int i = 0; i < NW; ++i) K.w[i] = __funnelshift_l(x[i + 1], x[i], s);
-    if (NW >= 2) K.w[NW - 2] &= m.m2;
-    K.w[NW - 1] &= m.m1;
-    return K;
-}
-__device__ __forceinline__ uint32_t base32s(uint32_t rowb, int i) {
-    return (lds32(rowb + 4u * (uint32_t)((i >> 4) ^ 1)) >> (30 - ((i & 15) << 1))) & 3u;
-}
-
 template <int NW, int UNR, bool SM = false, typename F>
 __device__ __forceinline__ void warp_positions32_dyn(const uint32_t *__restrict__ rseq, const uint32_t *__restrict__ rqc,
                                                      const uint8_t *__restrict__ rflag, uint32_t total, long long r0,

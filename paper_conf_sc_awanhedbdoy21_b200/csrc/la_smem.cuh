@@ -947,6 +947,9 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
             else if (LA_DYN && !GT && ulen > k)
                 warp_positions32_dyn<NW, UF>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop,
                                                            &B.ctr_f, filt);
+            else if (sreads && LA_LDS_READS)
+                warp_positions32<NW, UF, true>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
+                                               stop, filt);
             else
                 warp_positions32<NW, UF>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
                                                        stop, filt);
@@ -984,6 +987,9 @@ __device__ __forceinline__ void inl32_build_link(BuildCtl &B, const TabCtx &TC, 
                                               &B.ctr_b, build);
         else if (LA_DYN && !GT && ulen > k)
             warp_positions32_dyn<NW, 1>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref[r], r0, SW2, k, ulen, lane, stop, &B.ctr_b, build);
+        else if (sreads && LA_LDS_READS)
+            warp_positions32<NW, 1, true>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane,
+                                          stop, build);
         else
             warp_positions32<NW>(R32, Q32, ((LA_ANYN && !anyN) ? nullptr : rflag), pref, r0, r, SW2, k, ulen, wid, nwarps, lane, stop, build);
         flush_vote32(pend, &B.overflow);
@@ -1436,6 +1442,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
         // XL: stage this end's reads in shared memory when they fit beside the filter bitmaps (the
         // streamed reads were the XL kernel's top stall: long scoreboard on L2, ncu r01)
         SmemFixed FXt = FX;
+        bool xl_staged = false;   // XL: this end's reads staged in shared memory
         if (GT && !no_room) {
             const uint32_t xs = (stage_bytes(r, SW) + 127u) & ~127u;
             const uint32_t mw = ((4u * U + 31u) / 32u + 3u) & ~3u;
@@ -1456,6 +1463,7 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
                     xF[i] = __ldg(&rflag[r0 + i]);
                 }
                 builders_sync(NB);
+                xl_staged = true;
                 gR = xR;
                 gQ = xQ;
                 gL = xL;
@@ -1521,10 +1529,10 @@ __global__ void __launch_bounds__(BLOCK, MINB) k_smem(
             uint32_t *queue = (uint32_t *)(sm + FX.off_queue) + (bt >> 5) * 64;
             if (INL)
                 build_link<true, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, !GT && !stream);
+                                     t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, GT ? xl_staged : !stream);
             else
                 build_link<false, GT>(B, T, B1, B2, mbits, info, gQ, gL, gF, pref, lr0, r, P, tail_e, Tn, n0, n1, bt, NB,
-                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, !GT && !stream);
+                                      t_filter, t_build, P.replay != 0, ulen_now, fpos, queue, E.anyN != 0, GT ? xl_staged : !stream);
             ovf = B.overflow != 0;   // uniform: last written before build_link's last barrier
             if (bt == 0) s_acc[6] += B.dead0;
         }
